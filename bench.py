@@ -1,0 +1,340 @@
+#!/usr/bin/env python3
+"""Benchmark of the fused Im2col-Winograd hot path on B200 (one JSON line on rank 0).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config cfg2] [--impl ours|reference]
+
+Metric (BASELINE.json): direct-conv-equivalent TFLOPS = 2*N*P*Q*C*K*R*S / time
+(PAPER.md:3942-3946), fp32 NHWC; plus the roofline fraction of the dominant
+kernel (the fused tcgen05 kernel) against the measured B200 peak.
+
+One step = the whole hot path for one batch resident in HBM: the filter transform
+(i2cw_filter_transform) + the fused kernel (i2cw_conv2d_nhwc_pretransformed);
+both are C-ABI calls, the same two launches i2cw_conv2d_nhwc makes. L2 is flushed
+(a 256 MiB memset, outside the timed intervals) before every step. Timing: CUDA
+events on the launching stream around each call; the sum over K steps, max over
+ranks. Multi-GPU: torchrun, one rank per GPU, batch sharding with a FIXED per-GPU
+batch (weak scaling), no collective inside the timed region.
+`--impl reference` times the fp64 CPU oracle (the reference arm for this tier).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "direct-conv-equiv TFLOPS (fp32 NHWC, r=2..9) at 1/2/4/8 B200; % of roofline"
+
+# BASELINE.json configs; the headline (N=1 default) is configs[1], the ResNet-style 3x3 layer.
+CONFIGS = {
+    "cfg1": ("conv", 1, 8, 8, 4, 4, 3, 3, 1, 1, "N=1, H=W=8, C=K=4, 3x3, pad 1 fp32 NHWC conv (tiny)"),
+    "cfg2": ("conv", 128, 56, 56, 64, 64, 3, 3, 1, 1, "ResNet-style 3x3 layer: N=128, H=W=56, C=K=64, pad 1 fp32 NHWC conv"),
+    "cfg4-r5": ("deconv", 64, 28, 28, 256, 256, 5, 5, 2, 2, "deconv 5x5: N=64, H=W=28, C=K=256, pad 2"),
+    "cfg4-r7": ("deconv", 64, 28, 28, 256, 256, 7, 7, 3, 3, "deconv 7x7: N=64, H=W=28, C=K=256, pad 3"),
+    "cfg5a": ("conv", 256, 112, 112, 64, 64, 7, 7, 3, 3, "ILSVRC 7x7: N=256, H=W=112, C=K=64, pad 3"),
+}
+for _r in range(2, 10):
+    CONFIGS[f"cfg3-r{_r}"] = ("conv", 64, 32, 32, 128, 128, _r, _r, _r // 2, _r // 2,
+                              f"filter-width sweep r={_r}: N=64, H=W=32, C=K=128, pad {_r // 2}")
+for _c in (64, 128, 256, 512):
+    CONFIGS[f"cfg5b-c{_c}"] = ("conv", 256, 28, 28, _c, _c, 3, 3, 1, 1, f"ILSVRC 3x3: N=256, H=W=28, C=K={_c}, pad 1")
+
+
+def out_hw(kind, H, W, R, S, ph, pw):
+    if kind == "conv":
+        return H + 2 * ph - R + 1, W + 2 * pw - S + 1
+    return H + R - 1 - 2 * ph, W + S - 1 - 2 * pw
+
+
+def direct_flops(cfg, n_images=None):
+    kind, N, H, W, C, K, R, S, ph, pw, _ = cfg
+    P, Q = out_hw(kind, H, W, R, S, ph, pw)
+    return 2.0 * (N if n_images is None else n_images) * P * Q * C * K * R * S
+
+
+def load_peaks():
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(path) as f:
+            pk = json.load(f)
+        return pk, "measured"
+    except Exception:
+        return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0}, "fallback"
+
+
+class ClockSampler:
+    """NVML sampling of SM clock and throttle reasons while the timed region runs."""
+
+    REASONS = {"sw_power_cap": 0x4, "hw_slowdown": 0x8, "sw_thermal_slowdown": 0x20, "hw_thermal_slowdown": 0x40,
+               "hw_power_brake_slowdown": 0x80}
+
+    def __init__(self, device_index):
+        self.samples, self.reasons, self.max_mhz = [], set(), None
+        self._stop = threading.Event()
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(device_index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+        except Exception:
+            self.nv = None
+        self._t = threading.Thread(target=self._run, daemon=True)
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                r = self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                for k, bit in self.REASONS.items():
+                    if r & bit:
+                        self.reasons.add(k)
+            except Exception:
+                pass
+            time.sleep(0.002)
+
+    def __enter__(self):
+        if self.nv is not None:
+            self._t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self.nv is not None:
+            self._t.join()
+
+    def summary(self):
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons), "samples": 0}
+        return {"sm_mhz": statistics.median(self.samples), "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons),
+                "samples": len(self.samples)}
+
+
+def cpu_oracle_sample(cfg, budget_s=12.0, max_images=None):
+    """Time the fp64 oracle (y only) on a bounded sample of whole images of the workload."""
+    import oracle
+    from synthetic import make_w, make_x
+    kind, N, H, W, C, K, R, S, ph, pw, _ = cfg
+    w = make_w(K, R, S, C) if kind == "conv" else make_w(C, R, S, K)
+    f = oracle.conv2d_nhwc if kind == "conv" else oracle.deconv2d_nhwc
+    x1 = make_x(0, 1, H, W, C)
+    t0 = time.perf_counter()
+    f(x1, w, ph, pw, with_bound=False)
+    t1 = time.perf_counter() - t0
+    n = max(1, min(N if max_images is None else max_images, int(budget_s / max(t1, 1e-6))))
+    x = make_x(0, n, H, W, C)
+    t0 = time.perf_counter()
+    f(x, w, ph, pw, with_bound=False)
+    dt = time.perf_counter() - t0
+    return {"value": direct_flops(cfg, n) / dt / 1e12, "unit": "TFLOPS", "cores": oracle.num_threads(),
+            "kind": "oracle",
+            "sample": f"{n} of {N} images of {cfg[-1]} (plain fp64 C oracle, y only), {dt:.2f} s"}
+
+
+def run_reference(args, cfg):
+    """--impl reference: the fp64 CPU oracle as it stands, rank 0 only, on a bounded sample."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    import oracle
+    from synthetic import make_w, make_x
+    kind, N, H, W, C, K, R, S, ph, pw, desc = cfg
+    w = make_w(K, R, S, C) if kind == "conv" else make_w(C, R, S, K)
+    f = oracle.conv2d_nhwc if kind == "conv" else oracle.deconv2d_nhwc
+    x1 = make_x(0, 1, H, W, C)
+    t0 = time.perf_counter()
+    f(x1, w, ph, pw, with_bound=False)
+    t1 = time.perf_counter() - t0
+    # each step: the same whole-image sample, sized so the whole run stays within ~2-3 minutes
+    per_step_budget = 120.0 / max(1, args.steps + args.warmup)
+    n = max(1, min(N, int(per_step_budget / max(t1, 1e-6))))
+    x = make_x(0, n, H, W, C)
+    for _ in range(args.warmup):
+        f(x, w, ph, pw, with_bound=False)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        f(x, w, ph, pw, with_bound=False)
+    dt = (time.perf_counter() - t0) / args.steps
+    v = direct_flops(cfg, n) / dt / 1e12
+    sample = f"{n} of {N} images of the workload per step (plain fp64 C oracle, y only)"
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "TFLOPS", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt * 1e3, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": desc, "name": args.config, "images_per_step": n},
+            "cpu_baseline": {"value": v, "unit": "TFLOPS", "cores": oracle.num_threads(), "kind": "oracle",
+                             "sample": sample},
+            "e2e": {"value": v, "unit": "TFLOPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=100)
+    ap.add_argument("--warmup", type=int, default=10)
+    ap.add_argument("--config", default="cfg2", choices=sorted(CONFIGS))
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    ap.add_argument("--no-e2e", action="store_true", help="skip the host-buffer end-to-end leg")
+    ap.add_argument("--e2e-steps", type=int, default=10)
+    args = ap.parse_args()
+    if args.warmup < 3:
+        raise SystemExit("--warmup must be >= 3")
+    cfg = CONFIGS[args.config]
+    if args.impl == "reference":
+        run_reference(args, cfg)
+        return
+
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_icpp_zhangzxyw24_b200 as i2cw
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}")
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        dist.init_process_group("nccl", device_id=dev)
+
+    kind, N, H, W, C, K, R, S, ph, pw, desc = cfg
+    P, Q = out_hw(kind, H, W, R, S, ph, pw)
+    is_deconv = kind == "deconv"
+    # per-GPU batch fixed (weak scaling); images of rank r are global images r*N .. r*N+N-1
+    g = torch.Generator(device=dev).manual_seed(1000 + rank)
+    x = torch.rand((N, H, W, C), generator=g, device=dev).mul_(2).sub_(1)
+    g.manual_seed(7)
+    w = torch.rand((K, R, S, C) if not is_deconv else (C, R, S, K), generator=g, device=dev).mul_(2).sub_(1)
+    y = torch.empty((N, P, Q, K), device=dev)
+    u = torch.empty(i2cw.filter_bytes(C, K, R, S), dtype=torch.uint8, device=dev)
+    flush = torch.empty(64 * 1024 * 1024, dtype=torch.float32, device=dev)  # 256 MiB > 126 MB L2
+    stream = torch.cuda.current_stream()
+    L = i2cw.lib()
+    sp = stream.cuda_stream
+    conv_pre = L.i2cw_deconv2d_nhwc_pretransformed if is_deconv else L.i2cw_conv2d_nhwc_pretransformed
+
+    def step():
+        rc = L.i2cw_filter_transform(C, K, R, S, int(is_deconv), w.data_ptr(), u.data_ptr(), sp)
+        if rc:
+            raise i2cw.I2CWError("i2cw_filter_transform", rc)
+        ev_mid.record(stream)
+        rc = conv_pre(N, H, W, C, K, R, S, ph, pw, x.data_ptr(), u.data_ptr(), y.data_ptr(), sp)
+        if rc:
+            raise i2cw.I2CWError("i2cw_conv2d_nhwc_pretransformed", rc)
+
+    # warm-up (also validates the call path)
+    for _ in range(args.warmup):
+        flush.zero_()
+        ev_mid = torch.cuda.Event(enable_timing=True)
+        step()
+    torch.cuda.synchronize()
+
+    evs = [[torch.cuda.Event(enable_timing=True) for _ in range(3)] for _ in range(args.steps)]
+    sampler = ClockSampler(local)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    with sampler:
+        for i in range(args.steps):
+            flush.zero_()
+            e0, ev_mid, e2 = evs[i]
+            e0.record(stream)
+            step()
+            e2.record(stream)
+        torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    t_total = sum(e[0].elapsed_time(e[2]) for e in evs) / 1e3        # s, K steps
+    t_fused = sum(e[1].elapsed_time(e[2]) for e in evs) / 1e3
+    t_ft = sum(e[0].elapsed_time(e[1]) for e in evs) / 1e3
+    tt = torch.tensor([t_total, t_fused, t_ft], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+    t_total, t_fused, t_ft = tt.tolist()
+
+    # end-to-end through the public host-buffer call (H2D x, w + conv + D2H y every step)
+    e2e = None
+    if not args.no_e2e:
+        xh = x.cpu().pin_memory()
+        wh = w.cpu().pin_memory()
+        yh = torch.empty((N, P, Q, K)).pin_memory()
+        for _ in range(2):
+            i2cw.conv2d_nhwc_host(xh, wh, ph, pw, is_deconv=is_deconv, out=yh)
+        if world > 1:
+            dist.barrier()
+        ea, eb = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        torch.cuda.synchronize()
+        ea.record(stream)
+        for _ in range(args.e2e_steps):
+            i2cw.conv2d_nhwc_host(xh, wh, ph, pw, is_deconv=is_deconv, out=yh)
+        eb.record(stream)
+        torch.cuda.synchronize()
+        te = torch.tensor([ea.elapsed_time(eb) / 1e3], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(te, op=dist.ReduceOp.MAX)
+        e2e = {"value": direct_flops(cfg) * world * args.e2e_steps / te.item() / 1e12, "unit": "TFLOPS",
+               "h2d_bytes_per_step": (x.numel() + w.numel()) * 4, "d2h_bytes_per_step": y.numel() * 4,
+               "steps": args.e2e_steps, "api": "i2cw_conv2d_nhwc_host (pinned host buffers)"}
+
+    clocks = sampler.summary()
+    if rank == 0:
+        pk, pk_src = load_peaks()
+        p = i2cw.debug_plan(kind, N, H, W, C, K, R, S, ph, pw)
+        m, alpha = p["m"], p["alpha"]
+        # algorithmic tensor work of the fused kernel per launch: 3xTF32,
+        # fractional tiles per output row: F_tc = 3 * 2 * alpha * N * P * (Q/m) * K * R * C
+        f_tc = 3 * 2 * alpha * N * P * (Q / m) * K * R * C
+        t_fused_launch = t_fused / args.steps
+        tf32_peak = pk["bf16_tflops"] * 0.5  # tf32 dense = bf16 dense / 2 (nominal ratio)
+        achieved = f_tc / t_fused_launch / 1e12
+        # algorithmic HBM bytes of the fused kernel: x read once, y written once, U read once
+        hbm_bytes = 4 * (N * H * W * C + N * P * Q * K) + (i2cw.filter_bytes(C, K, R, S) - 256)
+        traffic = None
+        tpath = os.path.join(ROOT, "profiles", "traffic.json")
+        if os.path.exists(tpath):
+            try:
+                traffic = json.load(open(tpath)).get(args.config)
+            except Exception:
+                traffic = None
+        value = direct_flops(cfg) * world * args.steps / t_total / 1e12
+        line = {
+            "metric": METRIC, "value": value, "unit": "TFLOPS", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": t_total / args.steps * 1e3, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f32 (3xTF32 tcgen05 contraction)",
+            "data": "synthetic",
+            "config": {"workload": desc, "name": args.config, "per_gpu_batch": N, "global_batch": N * world,
+                       "parallelism": f"batch-sharded x{world}, no collective in the timed region",
+                       "F(m,r)": f"F({m},{S}) alpha={alpha}", "l2": "flushed (256 MiB memset) before every step",
+                       "step": "i2cw_filter_transform + i2cw_conv2d_nhwc_pretransformed (C ABI)"},
+            "roofline": {"bound": "tensor", "achieved": achieved, "peak": tf32_peak, "unit": "TFLOP/s",
+                         "frac": achieved / tf32_peak, "traffic": traffic,
+                         "kernel": "fused_tc_kernel", "kernel_ms": t_fused_launch * 1e3,
+                         "work": "3xTF32 UMMA flops 6*alpha*N*P*(Q/m)*K*R*C per launch",
+                         "peak_src": f"{pk_src}: bf16_tflops {pk['bf16_tflops']} x 0.5 (tf32/bf16 nominal)",
+                         "hbm_frac": hbm_bytes / t_fused_launch / 1e9 / pk["hbm_gbs"],
+                         "filter_transform_ms": t_ft / args.steps * 1e3},
+            "gpu_launches": 2 * args.steps,
+            "clocks": clocks,
+        }
+        if e2e is not None:
+            line["e2e"] = e2e
+        if world == 1 and not args.no_cpu:
+            line["cpu_baseline"] = cpu_oracle_sample(cfg)
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

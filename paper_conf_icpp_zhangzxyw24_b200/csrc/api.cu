@@ -1,0 +1,486 @@
+// C ABI (include/i2cw.h): argument validation, the host planner, TMA tensor-map
+// encoding, the stream-ordered workspace and the two launches per call
+// (filter transform, fused kernel).
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdint>
+#include <cstring>
+#include <mutex>
+#include <vector>
+
+#include "../../include/i2cw.h"
+#include "common.cuh"
+#include "cook_toom.h"
+
+namespace i2cw {
+cudaError_t launch_filter_transform(const float* w, float* u, int C, int K, int R, int S, int is_deconv, int alpha,
+                                    int NT, int NB, int NCC, const double* G, cudaStream_t stream);
+cudaError_t launch_fused_tc(const CUtensorMap& xmap, const Plan& pl, const float* u, float* y, cudaStream_t stream);
+cudaError_t launch_fused_simt(const Plan& pl, const float* x, const float* u, float* y, cudaStream_t stream);
+
+namespace {
+
+constexpr int kNWG = 2;                // transform warpgroups in the tc kernel
+constexpr int kSmemBudget = 225 * 1024;
+
+// Per filter width S: F(m, S) and the point set. r = 2..7 follow the paper's
+// Gamma_8 choices (Table 2). For r = 8, 9 the paper uses
+// Gamma_16; on B200 the tcgen05 fp32 accumulation measured max err/bound 1.1e-4
+// with alpha = 16 (alt points) > the 5e-5 acceptance of DESIGN.md reading R7,
+// so r = 8, 9 use alpha = 12 (F(5,8), F(4,9); paper point order). Setting
+// I2CW_ALPHA16=1 selects alpha = 16 (alt points) for r = 7..9 (ablation only).
+struct Choice { int m, alpha, point_set; };
+bool alpha16_override() {
+  static const bool on = [] { const char* e = getenv("I2CW_ALPHA16"); return e && e[0] == '1'; }();
+  return on;
+}
+bool choose(int S, Choice* c) {
+  if (alpha16_override() && S >= 7 && S <= 9) { *c = {17 - S, 16, 1}; return true; }
+  switch (S) {
+    case 2: *c = {7, 8, 0}; return true;
+    case 3: *c = {6, 8, 0}; return true;
+    case 4: *c = {5, 8, 0}; return true;
+    case 5: *c = {4, 8, 0}; return true;
+    case 6: *c = {3, 8, 0}; return true;
+    case 7: *c = {2, 8, 0}; return true;
+    case 8: *c = {5, 12, 0}; return true;
+    case 9: *c = {4, 12, 0}; return true;
+    default: return false;
+  }
+}
+
+inline int cdiv(int a, int b) { return (a + b - 1) / b; }
+
+// lane -> (row, tile) permutation: every 8 consecutive lanes (one LDS.128
+// quarter-warp wavefront) should start at distinct 16-byte bank groups,
+// i.e. distinct (row * WBOX + tw * m) mod 8. Greedy over residue buckets.
+// Returns the summed conflict degree (0 = conflict-free).
+int assign_lanes(int ROWS, int TS, int WBOX, int m, unsigned char* lrow, unsigned char* ltw) {
+  std::vector<std::pair<int, int>> bucket[8];
+  for (int r = 0; r < ROWS; ++r)
+    for (int t = 0; t < TS; ++t) bucket[(r * WBOX + t * m) % 8].push_back({r, t});
+  std::fill(lrow, lrow + kMaxLanes, 0xFF);
+  std::fill(ltw, ltw + kMaxLanes, 0);
+  int lane = 0, cost = 0;
+  const int total = ROWS * TS;
+  while (lane < total) {
+    int cnt[8] = {0};
+    int in_group = 0;
+    // first pass: distinct residues, fullest buckets first
+    int order[8];
+    for (int i = 0; i < 8; ++i) order[i] = i;
+    std::sort(order, order + 8, [&](int a, int b) { return bucket[a].size() > bucket[b].size(); });
+    for (int oi = 0; oi < 8 && in_group < 8 && lane < total; ++oi) {
+      auto& bk = bucket[order[oi]];
+      if (bk.empty()) continue;
+      lrow[lane] = (unsigned char)bk.back().first;
+      ltw[lane] = (unsigned char)bk.back().second;
+      bk.pop_back();
+      cnt[order[oi]]++;
+      ++lane; ++in_group;
+    }
+    // fill the rest of the group (conflicting)
+    while (in_group < 8 && lane < total) {
+      int best = -1;
+      for (int i = 0; i < 8; ++i)
+        if (!bucket[i].empty() && (best < 0 || bucket[i].size() > bucket[best].size())) best = i;
+      auto& bk = bucket[best];
+      lrow[lane] = (unsigned char)bk.back().first;
+      ltw[lane] = (unsigned char)bk.back().second;
+      bk.pop_back();
+      cnt[best]++;
+      ++lane; ++in_group;
+    }
+    int mx = 0;
+    for (int i = 0; i < 8; ++i) mx = std::max(mx, cnt[i]);
+    cost += mx - 1;
+  }
+  return cost;
+}
+
+}  // namespace
+
+// Build the launch plan. Returns I2CW_OK or an error code.
+int make_plan(int N, int H, int W, int C, int K, int R, int S, int pad_h, int pad_w, int is_deconv, Plan* out) {
+  Plan pl;
+  std::memset(&pl, 0, sizeof(pl));
+  if (N <= 0 || H <= 0 || W <= 0 || C <= 0 || K <= 0 || R <= 0 || S <= 0 || pad_h < 0 || pad_w < 0) return I2CW_EINVAL;
+  Choice ch;
+  if (!choose(S, &ch)) return I2CW_EUNSUPPORTED;
+  if (C % 4 != 0 || K % 4 != 0) return I2CW_EUNSUPPORTED;
+  pl.N = N; pl.H = H; pl.W = W; pl.C = C; pl.K = K; pl.R = R; pl.S = S;
+  if (is_deconv) {  // deconv(x, w, pad) == conv(x, rot180(w)^T, R-1-pad)
+    pl.pad_h = R - 1 - pad_h;
+    pl.pad_w = S - 1 - pad_w;
+  } else {
+    pl.pad_h = pad_h;
+    pl.pad_w = pad_w;
+  }
+  pl.P = H + 2 * pl.pad_h - R + 1;
+  pl.Q = W + 2 * pl.pad_w - S + 1;
+  if (pl.P < 1 || pl.Q < 1) return I2CW_EINVAL;
+  pl.m = ch.m;
+  pl.alpha = ch.alpha;
+  pl.NT = K > 32 ? 64 : 32;
+  pl.GP = gp_for(pl.alpha, pl.NT);
+  pl.NPASS = pl.alpha / pl.GP;
+  pl.NB = cdiv(K, pl.NT);
+  pl.NCC = cdiv(C, 8);
+  pl.NKS = pl.NCC * R;
+  pl.T_r = cdiv(pl.Q, pl.m);
+  // WBOX <= 256 (TMA box limit), leave 7 columns of slack for the bank search
+  const int ts_max = std::min(kMaxLanes, (256 - 7 - (S - 1)) / pl.m);
+  if (ts_max < 1) return I2CW_EUNSUPPORTED;
+  pl.TS = std::min(pl.T_r, ts_max);
+  pl.SEGS = cdiv(pl.T_r, pl.TS);
+  int rows = pl.SEGS == 1 ? std::max(1, kMaxLanes / pl.TS) : 1;
+  rows = std::min(rows, pl.P);
+  rows = std::min(rows, 256 - (R - 1));
+  if (rows < 1) return I2CW_EUNSUPPORTED;
+  const int ubytes = pl.GP * 2 * pl.NT * 32;
+  pl.NUS = 4;
+  const int wmin = pl.TS * pl.m + S - 1;
+  for (;;) {
+    // balance rows over the row blocks of an image
+    const int pb = cdiv(pl.P, rows);
+    const int rows_bal = cdiv(pl.P, pb);
+    pl.ROWS = rows_bal;
+    pl.PB = pb;
+    pl.HBOX = pl.ROWS + R - 1;
+    int best = -1, bestw = wmin;
+    for (int wb = wmin; wb <= std::min(256, wmin + 7); ++wb) {
+      unsigned char lr[kMaxLanes], lt[kMaxLanes];
+      const int c = assign_lanes(pl.ROWS, pl.TS, wb, pl.m, lr, lt);
+      if (best < 0 || c < best) { best = c; bestw = wb; }
+    }
+    pl.WBOX = bestw;
+    pl.BOXB = pl.HBOX * pl.WBOX * 16;
+    pl.PLANE = (pl.BOXB + 127) / 128 * 128;
+    const int bar_bytes = 8 * (2 * 2 + 2 * kNWG + 2 + 2 * pl.NUS) + 16;
+    pl.smem_bytes = pl.NUS * ubytes + 2 * 2 * pl.PLANE + bar_bytes;
+    if (pl.smem_bytes <= kSmemBudget) break;
+    if (pl.NUS > 2) { pl.NUS--; continue; }
+    if (rows > 1) { rows = rows / 2; continue; }
+    return I2CW_EUNSUPPORTED;
+  }
+  assign_lanes(pl.ROWS, pl.TS, pl.WBOX, pl.m, pl.lane_row, pl.lane_tw);
+  pl.tile_blocks = N * pl.PB * pl.SEGS;
+  *out = pl;
+  return I2CW_OK;
+}
+
+namespace {
+
+typedef CUresult (*PFN_encodeTiled_t)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                      const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                      CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+PFN_encodeTiled_t get_encode() {
+  static PFN_encodeTiled_t fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<PFN_encodeTiled_t>(p);
+  });
+  return fn;
+}
+
+// x: [N][H][W][C] fp32; box = 4 channels x WBOX columns x HBOX rows x 1 image
+int encode_x_map(const Plan& pl, const float* x, CUtensorMap* map) {
+  PFN_encodeTiled_t enc = get_encode();
+  if (!enc) return I2CW_ECUDA;
+  cuuint64_t dims[4] = {(cuuint64_t)pl.C, (cuuint64_t)pl.W, (cuuint64_t)pl.H, (cuuint64_t)pl.N};
+  cuuint64_t strides[3] = {(cuuint64_t)pl.C * 4, (cuuint64_t)pl.W * pl.C * 4, (cuuint64_t)pl.H * pl.W * pl.C * 4};
+  cuuint32_t box[4] = {4, (cuuint32_t)pl.WBOX, (cuuint32_t)pl.HBOX, 1};
+  cuuint32_t es[4] = {1, 1, 1, 1};
+  CUresult r = enc(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, const_cast<float*>(x), dims, strides, box, es,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS ? I2CW_OK : I2CW_EUNSUPPORTED;
+}
+
+void ensure_pool(int dev) {
+  static std::mutex mu;
+  static bool done[64] = {false};
+  std::lock_guard<std::mutex> lk(mu);
+  if (dev < 0 || dev >= 64 || done[dev]) return;
+  cudaMemPool_t pool;
+  if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+    uint64_t thr = UINT64_MAX;
+    cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+  }
+  done[dev] = true;
+}
+
+// Our statically linked runtime keeps its own "current device": follow the
+// device that owns the caller's pointer (multi-GPU ranks use device != 0).
+int bind_device_of(const void* p) {
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) { cudaGetLastError(); return I2CW_EINVAL; }
+  if (a.type != cudaMemoryTypeDevice && a.type != cudaMemoryTypeManaged) return I2CW_EINVAL;
+  int cur = -1;
+  cudaGetDevice(&cur);
+  if (cur != a.device && cudaSetDevice(a.device) != cudaSuccess) return I2CW_ECUDA;
+  ensure_pool(a.device);
+  return I2CW_OK;
+}
+
+// Host-side copy of the tags written by i2cw_filter_transform, so the
+// pre-transformed calls can validate u without a device-to-host sync.
+std::mutex g_reg_mu;
+std::vector<std::pair<const void*, UTag>> g_registry;
+void registry_put(const void* u, const UTag& t) {
+  std::lock_guard<std::mutex> lk(g_reg_mu);
+  for (auto& e : g_registry)
+    if (e.first == u) { e.second = t; return; }
+  if (g_registry.size() >= 4096) g_registry.erase(g_registry.begin());
+  g_registry.push_back({u, t});
+}
+bool registry_lookup(const void* u, UTag* t) {
+  std::lock_guard<std::mutex> lk(g_reg_mu);
+  for (auto& e : g_registry)
+    if (e.first == u) { *t = e.second; return true; }
+  return false;
+}
+
+inline bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
+
+// exact G of F(m, S), rows permuted to the internal point order, as doubles
+void g_internal(const Plan& pl, int point_set, std::vector<double>* G) {
+  Transforms T = cook_toom(pl.m, pl.S, point_set);
+  G->assign((size_t)pl.alpha * pl.S, 0.0);
+  for (int idx = 0; idx < pl.alpha; ++idx)
+    for (int s = 0; s < pl.S; ++s) (*G)[(size_t)idx * pl.S + s] = T.G[(size_t)point_of(idx, pl.alpha) * pl.S + s].to_double();
+}
+
+size_t u_data_bytes(const Plan& pl) { return (size_t)pl.NB * pl.NKS * pl.alpha * 2 * pl.NT * 8 * 4; }
+
+int transform_into(const Plan& pl, int is_deconv, const float* w, void* u, cudaStream_t stream) {
+  Choice ch;
+  choose(pl.S, &ch);
+  std::vector<double> G;
+  g_internal(pl, ch.point_set, &G);
+  UTag tag;
+  std::memset(&tag, 0, sizeof(tag));
+  tag.magic = kUMagic; tag.alpha = pl.alpha; tag.m = pl.m; tag.is_deconv = is_deconv;
+  tag.C = pl.C; tag.K = pl.K; tag.R = pl.R; tag.S = pl.S; tag.NT = pl.NT; tag.NB = pl.NB; tag.NCC = pl.NCC;
+  static_assert(sizeof(UTag) <= kUTagBytes, "tag");
+  if (cudaMemcpyAsync(u, &tag, sizeof(tag), cudaMemcpyHostToDevice, stream) != cudaSuccess) return I2CW_ECUDA;
+  registry_put(u, tag);
+  float* ud = reinterpret_cast<float*>(static_cast<uint8_t*>(u) + kUTagBytes);
+  if (launch_filter_transform(w, ud, pl.C, pl.K, pl.R, pl.S, is_deconv, pl.alpha, pl.NT, pl.NB, pl.NCC, G.data(),
+                              stream) != cudaSuccess)
+    return I2CW_ECUDA;
+  return I2CW_OK;
+}
+
+int run_fused(const Plan& pl, const float* x, const void* u, float* y, cudaStream_t stream) {
+  CUtensorMap map;
+  int rc = encode_x_map(pl, x, &map);
+  if (rc != I2CW_OK) return rc;
+  const float* ud = reinterpret_cast<const float*>(static_cast<const uint8_t*>(u) + kUTagBytes);
+  return launch_fused_tc(map, pl, ud, y, stream) == cudaSuccess ? I2CW_OK : I2CW_ECUDA;
+}
+
+int conv_common(int is_deconv, int N, int H, int W, int C, int K, int R, int S, int pad_h, int pad_w, const float* x,
+                const float* w, float* y, cudaStream_t stream, bool simt) {
+  if (!x || !w || !y) return I2CW_EINVAL;
+  if (!aligned16(x) || !aligned16(w) || !aligned16(y)) return I2CW_EINVAL;
+  Plan pl;
+  int rc = make_plan(N, H, W, C, K, R, S, pad_h, pad_w, is_deconv, &pl);
+  if (rc != I2CW_OK) return rc;
+  if ((rc = bind_device_of(x)) != I2CW_OK) return rc;
+  void* u = nullptr;
+  const size_t ub = kUTagBytes + u_data_bytes(pl);
+  if (cudaMallocAsync(&u, ub, stream) != cudaSuccess) { cudaGetLastError(); return I2CW_ECUDA; }
+  rc = transform_into(pl, is_deconv, w, u, stream);
+  if (rc == I2CW_OK) {
+    if (simt)
+      rc = launch_fused_simt(pl, x, reinterpret_cast<const float*>(static_cast<uint8_t*>(u) + kUTagBytes), y, stream) ==
+                   cudaSuccess
+               ? I2CW_OK
+               : I2CW_ECUDA;
+    else
+      rc = run_fused(pl, x, u, y, stream);
+  }
+  cudaFreeAsync(u, stream);
+  if (rc != I2CW_OK) cudaGetLastError();
+  return rc;
+}
+
+int pretransformed_common(int is_deconv, int N, int H, int W, int C, int K, int R, int S, int pad_h, int pad_w,
+                          const float* x, const void* u, float* y, cudaStream_t stream) {
+  if (!x || !u || !y) return I2CW_EINVAL;
+  if (!aligned16(x) || !aligned16(u) || !aligned16(y)) return I2CW_EINVAL;
+  Plan pl;
+  int rc = make_plan(N, H, W, C, K, R, S, pad_h, pad_w, is_deconv, &pl);
+  if (rc != I2CW_OK) return rc;
+  if ((rc = bind_device_of(x)) != I2CW_OK) return rc;
+  UTag tag;
+  if (!registry_lookup(u, &tag)) {  // not made by i2cw_filter_transform in this process: read the device tag
+    if (cudaMemcpyAsync(&tag, u, sizeof(tag), cudaMemcpyDeviceToHost, stream) != cudaSuccess ||
+        cudaStreamSynchronize(stream) != cudaSuccess) {
+      cudaGetLastError();
+      return I2CW_ECUDA;
+    }
+  }
+  if (tag.magic != kUMagic || (int)tag.is_deconv != is_deconv || (int)tag.C != C || (int)tag.K != K ||
+      (int)tag.R != R || (int)tag.S != S || (int)tag.alpha != pl.alpha || (int)tag.m != pl.m || (int)tag.NT != pl.NT)
+    return I2CW_EINVAL;
+  rc = run_fused(pl, x, u, y, stream);
+  if (rc != I2CW_OK) cudaGetLastError();
+  return rc;
+}
+
+}  // namespace
+}  // namespace i2cw
+
+using namespace i2cw;
+
+extern "C" {
+
+const char* i2cw_status_string(int s) {
+  switch (s) {
+    case I2CW_OK: return "ok";
+    case I2CW_EINVAL: return "invalid argument";
+    case I2CW_EUNSUPPORTED: return "unsupported shape";
+    case I2CW_ECUDA: return "CUDA error";
+    default: return "unknown status";
+  }
+}
+
+int i2cw_version(void) { return 100; }
+
+int i2cw_conv2d_nhwc(int N, int H, int W, int C, int K, int R, int S, int pad_h, int pad_w, const float* x,
+                     const float* w, float* y, i2cw_stream_t stream) {
+  return conv_common(0, N, H, W, C, K, R, S, pad_h, pad_w, x, w, y, (cudaStream_t)stream, false);
+}
+
+int i2cw_deconv2d_nhwc(int N, int H, int W, int C, int K, int R, int S, int pad_h, int pad_w, const float* x,
+                       const float* w, float* y, i2cw_stream_t stream) {
+  return conv_common(1, N, H, W, C, K, R, S, pad_h, pad_w, x, w, y, (cudaStream_t)stream, false);
+}
+
+size_t i2cw_filter_bytes(int C, int K, int R, int S) {
+  Plan pl;
+  // the filter-side plan fields do not depend on N, H, W or pad: plan a 1 x R x S map
+  if (make_plan(1, R, S, C, K, R, S, 0, 0, 0, &pl) != I2CW_OK) return 0;
+  return kUTagBytes + u_data_bytes(pl);
+}
+
+int i2cw_filter_transform(int C, int K, int R, int S, int is_deconv, const float* w, void* u, i2cw_stream_t stream) {
+  if (!w || !u || !aligned16(w) || !aligned16(u) || (is_deconv != 0 && is_deconv != 1)) return I2CW_EINVAL;
+  Plan pl;
+  int rc = make_plan(1, R, S, C, K, R, S, 0, 0, 0, &pl);
+  if (rc != I2CW_OK) return rc;
+  if ((rc = bind_device_of(w)) != I2CW_OK) return rc;
+  rc = transform_into(pl, is_deconv, w, u, (cudaStream_t)stream);
+  if (rc != I2CW_OK) cudaGetLastError();
+  return rc;
+}
+
+int i2cw_conv2d_nhwc_pretransformed(int N, int H, int W, int C, int K, int R, int S, int pad_h, int pad_w,
+                                    const float* x, const void* u, float* y, i2cw_stream_t stream) {
+  return pretransformed_common(0, N, H, W, C, K, R, S, pad_h, pad_w, x, u, y, (cudaStream_t)stream);
+}
+
+int i2cw_deconv2d_nhwc_pretransformed(int N, int H, int W, int C, int K, int R, int S, int pad_h, int pad_w,
+                                      const float* x, const void* u, float* y, i2cw_stream_t stream) {
+  return pretransformed_common(1, N, H, W, C, K, R, S, pad_h, pad_w, x, u, y, (cudaStream_t)stream);
+}
+
+int i2cw_set_device(int device) {
+  if (cudaSetDevice(device) != cudaSuccess) { cudaGetLastError(); return I2CW_ECUDA; }
+  ensure_pool(device);
+  return I2CW_OK;
+}
+
+int i2cw_conv2d_nhwc_host(int is_deconv, int N, int H, int W, int C, int K, int R, int S, int pad_h, int pad_w,
+                          const float* x_host, const float* w_host, float* y_host, i2cw_stream_t stream_) {
+  if (!x_host || !w_host || !y_host || (is_deconv != 0 && is_deconv != 1)) return I2CW_EINVAL;
+  cudaStream_t stream = (cudaStream_t)stream_;
+  Plan pl;
+  int rc = make_plan(N, H, W, C, K, R, S, pad_h, pad_w, is_deconv, &pl);
+  if (rc != I2CW_OK) return rc;
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) { cudaGetLastError(); return I2CW_ECUDA; }
+  ensure_pool(dev);
+  const size_t xb = (size_t)N * H * W * C * 4, wb = (size_t)K * R * S * C * 4, yb = (size_t)N * pl.P * pl.Q * K * 4;
+  float *xd = nullptr, *wd = nullptr, *yd = nullptr;
+  if (cudaMallocAsync(&xd, xb, stream) != cudaSuccess || cudaMallocAsync(&wd, wb, stream) != cudaSuccess ||
+      cudaMallocAsync(&yd, yb, stream) != cudaSuccess) {
+    cudaGetLastError();
+    if (xd) cudaFreeAsync(xd, stream);
+    if (wd) cudaFreeAsync(wd, stream);
+    return I2CW_ECUDA;
+  }
+  rc = I2CW_OK;
+  if (cudaMemcpyAsync(xd, x_host, xb, cudaMemcpyHostToDevice, stream) != cudaSuccess ||
+      cudaMemcpyAsync(wd, w_host, wb, cudaMemcpyHostToDevice, stream) != cudaSuccess)
+    rc = I2CW_ECUDA;
+  if (rc == I2CW_OK) rc = conv_common(is_deconv, N, H, W, C, K, R, S, pad_h, pad_w, xd, wd, yd, stream, false);
+  if (rc == I2CW_OK && cudaMemcpyAsync(y_host, yd, yb, cudaMemcpyDeviceToHost, stream) != cudaSuccess) rc = I2CW_ECUDA;
+  cudaFreeAsync(xd, stream);
+  cudaFreeAsync(wd, stream);
+  cudaFreeAsync(yd, stream);
+  if (cudaStreamSynchronize(stream) != cudaSuccess) rc = I2CW_ECUDA;
+  if (rc != I2CW_OK) cudaGetLastError();
+  return rc;
+}
+
+int i2cw_plan(int S, int* m, int* alpha, int* point_set) {
+  Choice c;
+  if (!choose(S, &c)) return I2CW_EUNSUPPORTED;
+  if (m) *m = c.m;
+  if (alpha) *alpha = c.alpha;
+  if (point_set) *point_set = c.point_set;
+  return I2CW_OK;
+}
+
+int i2cw_transform_matrices_rational(int m, int r, int point_set, int64_t* at_num, int64_t* at_den, int64_t* g_num,
+                                     int64_t* g_den, int64_t* bt_num, int64_t* bt_den) {
+  if (m < 1 || r < 1 || m + r - 1 > 16 || m + r - 1 < 2 || (point_set != 0 && point_set != 1)) return I2CW_EINVAL;
+  if (point_set == 1 && m + r - 1 != 16) return I2CW_EINVAL;
+  if (!at_num || !at_den || !g_num || !g_den || !bt_num || !bt_den) return I2CW_EINVAL;
+  Transforms T;
+  try {
+    T = cook_toom(m, r, point_set);
+  } catch (...) {
+    return I2CW_EUNSUPPORTED;
+  }
+  const i128 lim = (i128)INT64_MAX;
+  auto put = [&](const std::vector<Rat>& v, int64_t* num, int64_t* den) {
+    for (size_t i = 0; i < v.size(); ++i) {
+      if (v[i].n > lim || v[i].n < -lim || v[i].d > lim) return false;
+      num[i] = (int64_t)v[i].n;
+      den[i] = (int64_t)v[i].d;
+    }
+    return true;
+  };
+  if (!put(T.AT, at_num, at_den) || !put(T.G, g_num, g_den) || !put(T.BT, bt_num, bt_den)) return I2CW_EUNSUPPORTED;
+  return I2CW_OK;
+}
+
+// ---- not part of the public header: test hooks (csrc/debug_api.h) ----
+I2CW_API int i2cw_debug_conv_simt(int is_deconv, int N, int H, int W, int C, int K, int R, int S, int pad_h, int pad_w,
+                         const float* x, const float* w, float* y, i2cw_stream_t stream) {
+  return conv_common(is_deconv, N, H, W, C, K, R, S, pad_h, pad_w, x, w, y, (cudaStream_t)stream, true);
+}
+
+I2CW_API int i2cw_debug_plan(int is_deconv, int N, int H, int W, int C, int K, int R, int S, int pad_h, int pad_w,
+                    int* out /* 32 ints */) {
+  Plan pl;
+  int rc = make_plan(N, H, W, C, K, R, S, pad_h, pad_w, is_deconv, &pl);
+  if (rc != I2CW_OK) return rc;
+  int v[] = {pl.P, pl.Q, pl.m, pl.alpha, pl.NT, pl.NB, pl.NCC, pl.NKS, pl.T_r, pl.TS, pl.SEGS, pl.ROWS, pl.PB,
+             pl.WBOX, pl.HBOX, pl.tile_blocks, pl.GP, pl.NPASS, pl.NUS, pl.smem_bytes, pl.pad_h, pl.pad_w};
+  for (int i = 0; i < 32; ++i) out[i] = i < (int)(sizeof(v) / sizeof(v[0])) ? v[i] : 0;
+  return I2CW_OK;
+}
+
+}  // extern "C"

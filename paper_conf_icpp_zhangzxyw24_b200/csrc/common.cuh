@@ -1,0 +1,218 @@
+// Shared definitions for the i2cw CUDA path: the launch plan (host-computed,
+// passed by value) and thin inline-PTX wrappers for sm_100a mbarrier, TMA /
+// bulk copies and tcgen05 (TMEM alloc, MMA, ld/st, commit, fences).
+#pragma once
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace i2cw {
+
+constexpr int kMaxLanes = 128;  // UMMA M = 128 Winograd tiles per CTA (one TMEM lane each)
+
+// Everything the kernels need about one call; built by make_plan() in api.cu.
+struct Plan {
+  int N, H, W, C, K, R, S;
+  int pad_h, pad_w;     // conv padding as seen by the kernel (deconv: R-1-pad, may be < 0)
+  int P, Q;             // output height / width
+  int m, alpha;         // F(m, S), alpha = m + S - 1
+  int NT;               // output channels per CTA (UMMA N)
+  int NB;               // ceil(K / NT)
+  int NCC;              // ceil(C / 8) channel chunks (8 fp32 = one tf32 UMMA K step)
+  int NKS;              // k-steps = NCC * R  (ks = cc * R + fh)
+  int T_r;              // Winograd tiles per output row = ceil(Q / m)
+  int TS;               // tiles per row segment handled by one CTA
+  int SEGS;             // segments per row = ceil(T_r / TS)
+  int ROWS;             // output rows per CTA
+  int PB;               // row blocks per image = ceil(P / ROWS)
+  int WBOX, HBOX;       // staged input box (columns, rows = ROWS + R - 1)
+  int BOXB;             // bytes of one TMA box (one 4-channel plane) = HBOX*WBOX*16
+  int PLANE;            // shared-memory stride between planes (BOXB rounded up to 128)
+  int tile_blocks;      // N * PB * SEGS
+  int GP, NPASS;        // points per pass (TMEM budget), passes = alpha / GP
+  int NUS;              // U pipeline stages
+  int smem_bytes;
+  unsigned char lane_row[kMaxLanes];  // lane -> row within block (0xFF = idle lane)
+  unsigned char lane_tw[kMaxLanes];   // lane -> tile within segment
+};
+
+// Points per TMEM pass: GP * NT accumulator columns + 2 V stages of GP * 16
+// columns <= 512, GP even and dividing alpha.
+__host__ __device__ constexpr int gp_for(int alpha, int NT) {
+  return NT == 64 ? 4 : (alpha % 8 == 0 ? 8 : 6);
+}
+
+// Internal Winograd point order: singles {0, alpha-1} first, then the ± pairs
+// (1,2), (3,4), ... so that every pass of GP (even) points holds whole pairs
+// (PAPER.md:595-603 pair structure).
+__host__ __device__ constexpr int point_of(int idx, int alpha) {
+  return idx == 0 ? 0 : (idx == 1 ? alpha - 1 : idx - 1);
+}
+
+// U (transformed filter) layout, fp32 words:
+//   U[nb][ks][idx][hl][kc][n][e],  idx = internal point index, hl = 0 hi / 1 lo,
+//   kc = 16-byte half of the 8-channel k-step, n < NT, e < 4  (channel = cc*8 + kc*4 + e)
+// i.e. one k-step's image for one (point, hl) is the UMMA K-major SWIZZLE_NONE
+// canonical layout of an NT x 8 tf32 tile with SBO = 128 B, LBO = NT * 16 B.
+__host__ __device__ inline size_t u_offset(int NT, int alpha, int nb, int NKS, int ks, int idx, int hl) {
+  return ((((size_t)nb * NKS + ks) * alpha + idx) * 2 + hl) * (size_t)NT * 8;
+}
+
+constexpr int kUTagBytes = 256;
+constexpr uint32_t kUMagic = 0x49324357u;  // "I2CW"
+struct UTag {
+  uint32_t magic, alpha, m, is_deconv, C, K, R, S, NT, NB, NCC, pad;
+};
+
+#if defined(__CUDACC__)
+// ----------------------------------------------------------------------------
+// PTX helpers
+// ----------------------------------------------------------------------------
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+__device__ __forceinline__ uint64_t globaltimer() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void fence_mbar_init() {
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ bool mbar_try_wait(uint64_t* bar, uint32_t parity) {
+  uint32_t ok;
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+      "selp.u32 %0, 1, 0, p;\n\t}"
+      : "=r"(ok)
+      : "r"(smem_u32(bar)), "r"(parity)
+      : "memory");
+  return ok != 0;
+}
+// Blocking wait with a watchdog: a protocol bug traps (launch error) after ~4 s
+// instead of hanging the GPU.
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  if (mbar_try_wait(bar, parity)) return;
+  const uint64_t t0 = globaltimer();
+  while (!mbar_try_wait(bar, parity)) {
+    if (globaltimer() - t0 > 4000000000ull) __trap();
+  }
+}
+
+// TMA: 4D tiled tensor load global -> shared, completes on an mbarrier (tx bytes)
+__device__ __forceinline__ void tma_load_4d(void* smem_dst, const CUtensorMap* map, uint64_t* bar, int c0, int c1,
+                                            int c2, int c3) {
+  asm volatile(
+      "cp.async.bulk.tensor.4d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+      " [%0], [%1, {%2, %3, %4, %5}], [%6];" ::"r"(smem_u32(smem_dst)),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "r"(smem_u32(bar))
+      : "memory");
+}
+__device__ __forceinline__ void tma_prefetch_desc(const CUtensorMap* map) {
+  asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(map)) : "memory");
+}
+// 1D bulk copy global -> shared (16-byte multiple), completes on an mbarrier
+__device__ __forceinline__ void bulk_load(void* smem_dst, const void* gsrc, uint32_t bytes, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(smem_dst)),
+      "l"(gsrc), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+
+// ---- tcgen05 --------------------------------------------------------------
+__device__ __forceinline__ void tmem_alloc(uint32_t* smem_dst, uint32_t ncols) {
+  asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(smem_dst)),
+               "r"(ncols)
+               : "memory");
+}
+__device__ __forceinline__ void tmem_relinquish() {
+  asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+}
+__device__ __forceinline__ void tmem_dealloc(uint32_t taddr, uint32_t ncols) {
+  asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(taddr), "r"(ncols) : "memory");
+}
+__device__ __forceinline__ void tc_fence_before() {
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+}
+__device__ __forceinline__ void tc_fence_after() {
+  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+}
+// D[tmem] (+)= A[tmem] * B[smem]^T, kind::tf32, M=128, N from idesc, K=8
+__device__ __forceinline__ void mma_tf32_ts(uint32_t d_tmem, uint32_t a_tmem, uint64_t b_desc, uint32_t idesc,
+                                            uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::1.kind::tf32 [%0], [%1], %2, %3, p;\n\t}" ::"r"(d_tmem),
+      "r"(a_tmem), "l"(b_desc), "r"(idesc), "r"(accumulate)
+      : "memory");
+}
+// D[tmem] (+)= A[smem] * B[smem]^T
+__device__ __forceinline__ void mma_tf32_ss(uint32_t d_tmem, uint64_t a_desc, uint64_t b_desc, uint32_t idesc,
+                                            uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem),
+      "l"(a_desc), "l"(b_desc), "r"(idesc), "r"(accumulate)
+      : "memory");
+}
+__device__ __forceinline__ void mma_commit(uint64_t* bar) {
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(smem_u32(bar))
+               : "memory");
+}
+__device__ __forceinline__ void tmem_st_x4(uint32_t taddr, float a, float b, float c, float d) {
+  asm volatile("tcgen05.st.sync.aligned.32x32b.x4.b32 [%0], {%1, %2, %3, %4};" ::"r"(taddr), "r"(__float_as_uint(a)),
+               "r"(__float_as_uint(b)), "r"(__float_as_uint(c)), "r"(__float_as_uint(d))
+               : "memory");
+}
+__device__ __forceinline__ void tmem_wait_st() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
+__device__ __forceinline__ void tmem_ld_x8(uint32_t taddr, float* v) {
+  uint32_t r[8];
+  asm volatile("tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"
+               : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7])
+               : "r"(taddr)
+               : "memory");
+#pragma unroll
+  for (int i = 0; i < 8; ++i) v[i] = __uint_as_float(r[i]);
+}
+__device__ __forceinline__ void tmem_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
+
+// tf32 round-to-nearest (ties away): the hi part of the 3xTF32 split
+__device__ __forceinline__ float tf32_rna(float x) {
+  uint32_t r;
+  asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(r) : "f"(x));
+  return __uint_as_float(r);
+}
+
+// UMMA shared-memory descriptor, K-major, SWIZZLE_NONE (canonical interleaved
+// layout: 8-row x 16-byte core matrices; SBO = byte stride between 8-row
+// groups, LBO = byte stride between the two 16-byte K halves).
+__device__ __forceinline__ uint64_t umma_desc_kmajor_noswizzle(uint32_t smem_addr, uint32_t lbo, uint32_t sbo) {
+  uint64_t d = 0;
+  d |= (uint64_t)((smem_addr >> 4) & 0x3FFFu);
+  d |= (uint64_t)((lbo >> 4) & 0x3FFFu) << 16;
+  d |= (uint64_t)((sbo >> 4) & 0x3FFFu) << 32;
+  d |= (uint64_t)1 << 46;  // descriptor version (sm_100)
+  return d;                // base offset 0, lbo mode 0, layout type 0 (no swizzle)
+}
+// Instruction descriptor for kind::tf32: D f32, A/B tf32, both K-major, M=128
+__host__ __device__ constexpr uint32_t idesc_tf32(int M, int N) {
+  return (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
+}
+#endif  // __CUDACC__
+
+}  // namespace i2cw

@@ -1,0 +1,70 @@
+// Filter transform U = G w (row a1 of SURVEY.md §8(a)).
+//
+// PAPER.md Alg 1 loadTiles (lines 355-362): G_tile = G(alpha,r) W_tile; §5.1
+// (534-541): forward filters are re-laid out for vector loads, and for the
+// backward deconvolution "the 180-degree filter-rotation is integrated into
+// filter-transformation" (no separate rearrangement pass).
+//
+// For every output-channel block nb, k-step ks = (cc, fh), internal point idx:
+//   U[nb][ks][idx][hl][kc][n][e] = split_hl( sum_s G[point(idx)][s] * w'(k, fh, s, c) )
+//   k = nb*NT + n, c = cc*8 + kc*4 + e (zero outside [0,K) x [0,C))
+//   conv:   w'(k, fh, s, c) = w[k][fh][s][c]                      (w is [K][R][S][C])
+//   deconv: w'(k, fh, s, c) = w[c][R-1-fh][S-1-s][k]              (w is [C][R][S][K])
+// G is applied in fp64 and rounded once to fp32 (the filter
+// transform's precision hardly matters); hi = tf32_rna(u), lo = tf32_rna(u - hi).
+#include "common.cuh"
+
+namespace i2cw {
+
+struct GTable {
+  double g[16 * 9];  // row = INTERNAL point index, col = tap s
+};
+
+__global__ void filter_transform_kernel(const float* __restrict__ w, float* __restrict__ u, int C, int K, int R,
+                                        int S, int is_deconv, int alpha, int NT, int NB, int NCC, GTable gt) {
+  const int NKS = NCC * R;
+  const size_t total = (size_t)NB * NKS * alpha * 2 * NT * 4;  // (nb, ks, idx, kc, n, e)
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < total; i += (size_t)gridDim.x * blockDim.x) {
+    size_t t = i;
+    const int e = (int)(t % 4); t /= 4;
+    const int n = (int)(t % NT); t /= NT;
+    const int kc = (int)(t % 2); t /= 2;
+    const int idx = (int)(t % alpha); t /= alpha;
+    const int ks = (int)(t % NKS); t /= NKS;
+    const int nb = (int)t;
+    const int cc = ks / R, fh = ks % R;
+    const int k = nb * NT + n, c = cc * 8 + kc * 4 + e;
+    float hi = 0.f, lo = 0.f;
+    if (k < K && c < C) {
+      double acc = 0.0;
+      for (int s = 0; s < S; ++s) {
+        const float wv = is_deconv ? w[(((size_t)c * R + (R - 1 - fh)) * S + (S - 1 - s)) * K + k]
+                                   : w[(((size_t)k * R + fh) * S + s) * C + c];
+        acc += gt.g[idx * 9 + s] * (double)wv;
+      }
+      const float uv = (float)acc;
+      hi = tf32_rna(uv);
+      lo = tf32_rna(uv - hi);
+    }
+    const size_t base = u_offset(NT, alpha, nb, NKS, ks, idx, 0) + (size_t)kc * NT * 4 + (size_t)n * 4 + e;
+    u[base] = hi;
+    u[base + (size_t)NT * 8] = lo;  // hl = 1 image follows the hl = 0 image
+  }
+}
+
+cudaError_t launch_filter_transform(const float* w, float* u, int C, int K, int R, int S, int is_deconv, int alpha,
+                                    int NT, int NB, int NCC, const double* G /* alpha x S, internal order */,
+                                    cudaStream_t stream) {
+  GTable gt;
+  for (int i = 0; i < 16 * 9; ++i) gt.g[i] = 0.0;
+  for (int i = 0; i < alpha; ++i)
+    for (int s = 0; s < S; ++s) gt.g[i * 9 + s] = G[i * S + s];
+  const size_t total = (size_t)NB * NCC * R * alpha * 2 * NT * 4;
+  int blocks = (int)((total + 255) / 256);
+  if (blocks > 148 * 16) blocks = 148 * 16;
+  if (blocks < 1) blocks = 1;
+  filter_transform_kernel<<<blocks, 256, 0, stream>>>(w, u, C, K, R, S, is_deconv, alpha, NT, NB, NCC, gt);
+  return cudaGetLastError();
+}
+
+}  // namespace i2cw

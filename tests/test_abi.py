@@ -1,0 +1,96 @@
+"""Host-side checks of the C ABI library (-m "not gpu"): it loads, exports every
+symbol include/i2cw.h declares, its host Cook-Toom generator matches the oracle's
+exactly, its planner is self-consistent, and bad arguments are rejected before
+any CUDA call. No GPU compute is invoked here."""
+import ctypes
+import os
+import re
+
+import pytest
+
+import paper_conf_icpp_zhangzxyw24_b200 as i2cw
+from oracle.cook_toom import cook_toom
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def header_symbols():
+    txt = open(os.path.join(ROOT, "include", "i2cw.h")).read()
+    return sorted(set(re.findall(r"I2CW_API\s+[\w\s\*]*?\b(i2cw_\w+)\s*\(", txt)))
+
+
+def test_library_exports_every_header_symbol():
+    syms = header_symbols()
+    assert len(syms) >= 12
+    assert sorted(i2cw.PUBLIC_SYMBOLS) == syms
+    L = ctypes.CDLL(i2cw.LIB_PATH)
+    for s in syms:
+        assert hasattr(L, s), s
+    assert i2cw.lib().i2cw_version() == 100
+    assert i2cw.status_string(-2) == "unsupported shape"
+
+
+PAIRS = [(7, 2), (6, 3), (5, 4), (4, 5), (3, 6), (2, 7), (10, 7), (9, 8), (8, 9), (6, 7), (5, 8), (4, 9), (3, 2),
+         (2, 3), (1, 4), (15, 2)]
+
+
+@pytest.mark.parametrize("m,r", PAIRS)
+def test_host_generator_matches_oracle_generator_exactly(m, r):
+    sets = ["paper"] + (["alt"] if m + r - 1 == 16 else [])
+    for ps in sets:
+        got = i2cw.transform_matrices(m, r, 0 if ps == "paper" else 1)
+        exp = cook_toom(m, r, ps)
+        assert got == tuple(exp) or list(got) == list(exp)
+
+
+def test_plan_table():
+    # paper's Table 2 Gamma_8 choices for r=2..7; r=8,9 alpha=12 (reading R7: alpha=16
+    # measured 1.1e-4 max err/bound on the tcgen05 accumulator, above the 5e-5 acceptance)
+    exp = {2: (7, 8, 0), 3: (6, 8, 0), 4: (5, 8, 0), 5: (4, 8, 0), 6: (3, 8, 0), 7: (2, 8, 0), 8: (5, 12, 0),
+           9: (4, 12, 0)}
+    for S, v in exp.items():
+        assert i2cw.plan(S) == v
+    with pytest.raises(i2cw.I2CWError):
+        i2cw.plan(10)
+
+
+CFGS = [("conv", 1, 8, 8, 4, 4, 3, 3, 1, 1), ("conv", 128, 56, 56, 64, 64, 3, 3, 1, 1),
+        ("deconv", 64, 28, 28, 256, 256, 5, 5, 2, 2), ("deconv", 64, 28, 28, 256, 256, 7, 7, 3, 3),
+        ("conv", 256, 112, 112, 64, 64, 7, 7, 3, 3), ("conv", 256, 28, 28, 512, 512, 3, 3, 1, 1)] + \
+       [("conv", 64, 32, 32, 128, 128, r, r, r // 2, r // 2) for r in range(2, 10)] + \
+       [("conv", 2, 5, 300, 8, 12, 2, 9, 0, 8), ("deconv", 3, 9, 13, 12, 20, 4, 3, 5, 0)]
+
+
+@pytest.mark.parametrize("cfg", CFGS)
+def test_planner_consistency(cfg):
+    kind, N, H, W, C, K, R, S, ph, pw = cfg
+    p = i2cw.debug_plan(kind, N, H, W, C, K, R, S, ph, pw)
+    P, Q = i2cw.out_shape(kind, N, H, W, K, R, S, ph, pw)[1:3]
+    assert (p["P"], p["Q"]) == (P, Q)
+    assert p["alpha"] == p["m"] + S - 1 and (p["m"], p["alpha"]) == i2cw.plan(S)[:2]
+    assert p["T_r"] == -(-Q // p["m"])
+    assert p["TS"] * p["SEGS"] >= p["T_r"] and p["ROWS"] * p["PB"] >= P
+    assert p["ROWS"] * p["TS"] <= 128
+    assert p["WBOX"] >= p["TS"] * p["m"] + S - 1 and p["WBOX"] <= 256 and p["HBOX"] == p["ROWS"] + R - 1
+    assert p["GP"] * p["NPASS"] == p["alpha"] and p["GP"] * p["NT"] + 2 * 16 * p["GP"] <= 512
+    assert p["NB"] * p["NT"] >= K and p["NCC"] * 8 >= C
+    assert p["smem_bytes"] <= 227 * 1024
+    assert p["tile_blocks"] == N * p["PB"] * p["SEGS"]
+
+
+def test_invalid_arguments_rejected_before_cuda():
+    L = i2cw.lib()
+    fake = 1 << 20  # non-null, 16-byte aligned (never dereferenced: validation fails first)
+    args = lambda **kw: [kw.get(k, v) for k, v in dict(N=1, H=8, W=8, C=8, K=8, R=3, S=3, ph=1, pw=1).items()]
+    assert L.i2cw_conv2d_nhwc(*args(S=10), fake, fake, fake, None) == i2cw.I2CW_EUNSUPPORTED
+    assert L.i2cw_conv2d_nhwc(*args(S=1), fake, fake, fake, None) == i2cw.I2CW_EUNSUPPORTED
+    assert L.i2cw_conv2d_nhwc(*args(C=6), fake, fake, fake, None) == i2cw.I2CW_EUNSUPPORTED
+    assert L.i2cw_conv2d_nhwc(*args(K=10), fake, fake, fake, None) == i2cw.I2CW_EUNSUPPORTED
+    assert L.i2cw_conv2d_nhwc(*args(N=0), fake, fake, fake, None) == i2cw.I2CW_EINVAL
+    assert L.i2cw_conv2d_nhwc(*args(ph=-1), fake, fake, fake, None) == i2cw.I2CW_EINVAL
+    assert L.i2cw_conv2d_nhwc(*args(H=1, ph=0), fake, fake, fake, None) == i2cw.I2CW_EINVAL  # P < 1
+    assert L.i2cw_conv2d_nhwc(*args(), None, fake, fake, None) == i2cw.I2CW_EINVAL
+    assert L.i2cw_conv2d_nhwc(*args(), fake + 4, fake, fake, None) == i2cw.I2CW_EINVAL  # misaligned
+    assert L.i2cw_deconv2d_nhwc(*args(S=12), fake, fake, fake, None) == i2cw.I2CW_EUNSUPPORTED
+    assert L.i2cw_filter_bytes(8, 8, 3, 11) == 0
+    assert L.i2cw_filter_bytes(64, 64, 3, 3) == 256 + 2 * 8 * 64 * 3 * 64 * 4

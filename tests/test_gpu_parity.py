@@ -1,0 +1,136 @@
+"""GPU parity: the tcgen05 path (through the C ABI) vs the fp64 oracle, element by
+element, |err| <= 1e-4 * sum|x||w| (BASELINE.json north_star). Sizes span several
+CTA tile blocks, ragged width tails (Q % m), partial output-channel blocks, padded
+channel chunks, multi-segment rows, every r = 2..9, conv and deconv."""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import paper_conf_icpp_zhangzxyw24_b200 as i2cw
+from tests.gpu_util import assert_parity, inputs, run_case
+
+pytestmark = pytest.mark.gpu
+
+RS = list(range(2, 10))
+
+
+def test_cfg1_tiny():
+    y, yr, b = run_case("conv", 1, 8, 8, 4, 4, 3, 3, 1, 1)
+    assert_parity(y, yr, b)
+
+
+@pytest.mark.parametrize("r", RS)
+@pytest.mark.parametrize("kind", ["conv", "deconv"])
+def test_r_sweep_same_pad(kind, r):
+    # K=40 > 32 -> NT=64 path with a partial channel block; W=37 ragged against every m
+    y, yr, b = run_case(kind, 2, 13, 37, 16, 40, r, r, r // 2, r // 2)
+    assert_parity(y, yr, b)
+
+
+@pytest.mark.parametrize("r", RS)
+@pytest.mark.parametrize("kind", ["conv", "deconv"])
+def test_r_sweep_small_k_nt32(kind, r):
+    # K=12 <= 32 -> NT=32 / GP=8 path; C=12 -> a half-empty second channel chunk
+    y, yr, b = run_case(kind, 3, 11, 23, 12, 12, r, r, r - 1, 0)
+    assert_parity(y, yr, b)
+
+
+@pytest.mark.parametrize("r", [3, 5, 8])
+@pytest.mark.parametrize("pad", ["zero", "max"])
+def test_pads(r, pad):
+    p = 0 if pad == "zero" else r - 1
+    for kind in ("conv", "deconv"):
+        y, yr, b = run_case(kind, 2, 12, 29, 8, 36, r, r, p, p)
+        assert_parity(y, yr, b)
+
+
+def test_deconv_pad_beyond_filter():
+    # pad > R-1: negative effective conv pad (a coordinate offset, reading R5)
+    y, yr, b = run_case("deconv", 2, 15, 21, 8, 8, 3, 5, 3, 5)
+    assert_parity(y, yr, b)
+
+
+@pytest.mark.parametrize("R,S", [(1, 3), (2, 5), (5, 3), (7, 2), (9, 4), (3, 9)])
+def test_rect_filters(R, S):
+    for kind in ("conv", "deconv"):
+        y, yr, b = run_case(kind, 2, 10, 27, 8, 20, R, S, R // 2, S // 2)
+        assert_parity(y, yr, b)
+
+
+@pytest.mark.parametrize("W", list(range(30, 36)))
+def test_width_residues_r3(W):
+    # Q = W with pad 1: Q % 6 takes every residue
+    y, yr, b = run_case("conv", 1, 9, W, 8, 64, 3, 3, 1, 1)
+    assert_parity(y, yr, b)
+
+
+def test_multi_segment_rows():
+    # Q = 308 with m = 8 -> 39 tiles per row, more than one CTA segment per row
+    p = i2cw.debug_plan("conv", 2, 5, 300, 8, 12, 2, 9, 0, 8)
+    assert p["SEGS"] > 1
+    y, yr, b = run_case("conv", 2, 5, 300, 8, 12, 2, 9, 0, 8)
+    assert_parity(y, yr, b)
+
+
+def test_many_channels_and_blocks():
+    y, yr, b = run_case("conv", 2, 9, 17, 136, 200, 3, 3, 1, 1)
+    assert_parity(y, yr, b)
+
+
+@pytest.mark.parametrize("r", [3, 7, 9])
+def test_simt_stepping_stone_matches_oracle(r):
+    for kind in ("conv", "deconv"):
+        y, yr, b = run_case(kind, 2, 11, 26, 8, 40, r, r, r // 2, r // 2, impl="simt")
+        assert_parity(y, yr, b)
+
+
+def test_pretransformed_filter_paths():
+    for kind, r in (("conv", 3), ("deconv", 5), ("conv", 9)):
+        x, w = inputs(kind, 2, 12, 20, 16, 24, r, r)
+        xd, wd = x.cuda(), w.cuda()
+        u = i2cw.filter_transform(wd, is_deconv=(kind == "deconv"))
+        K = w.shape[0] if kind == "conv" else w.shape[3]
+        y = i2cw.conv2d_nhwc_pretransformed(xd, u, K, r, r, r // 2, r // 2, is_deconv=(kind == "deconv"))
+        y1 = (i2cw.conv2d_nhwc if kind == "conv" else i2cw.deconv2d_nhwc)(xd, wd, r // 2, r // 2)
+        torch.cuda.synchronize()
+        assert torch.equal(y, y1)  # same kernels, same U -> bitwise equal
+        yr, b = (oracle.conv2d_nhwc if kind == "conv" else oracle.deconv2d_nhwc)(x, w, r // 2, r // 2)
+        assert_parity(y, yr, b)
+        # a u made for the other direction is rejected
+        with pytest.raises(i2cw.I2CWError):
+            i2cw.conv2d_nhwc_pretransformed(xd, u, K, r, r, r // 2, r // 2, is_deconv=(kind != "deconv"))
+
+
+def test_host_end_to_end_call():
+    x, w = inputs("conv", 2, 14, 19, 8, 16, 5, 5)
+    y = i2cw.conv2d_nhwc_host(x.pin_memory(), w.pin_memory(), 2, 2)
+    yr, b = oracle.conv2d_nhwc(x, w, 2, 2)
+    assert_parity(y, yr, b)
+    x, w = inputs("deconv", 2, 14, 19, 8, 16, 7, 7)
+    y = i2cw.conv2d_nhwc_host(x, w, 3, 3, is_deconv=True)
+    yr, b = oracle.deconv2d_nhwc(x, w, 3, 3)
+    assert_parity(y, yr, b)
+
+
+def test_deterministic_and_deconv_equals_flipped_conv():
+    x, w = inputs("deconv", 2, 13, 22, 16, 24, 5, 5)
+    xd, wd = x.cuda(), w.cuda()
+    y1 = i2cw.deconv2d_nhwc(xd, wd, 1, 2)
+    y2 = i2cw.deconv2d_nhwc(xd, wd, 1, 2)
+    torch.cuda.synchronize()
+    assert torch.equal(y1, y2)  # run-to-run bitwise determinism (no atomics)
+    wf = wd.flip(1).flip(2).permute(3, 1, 2, 0).contiguous()  # w'[k][r][s][c] = w[c][R-1-r][S-1-s][k]
+    yc = i2cw.conv2d_nhwc(xd, wf, 5 - 1 - 1, 5 - 1 - 2)
+    torch.cuda.synchronize()
+    _, b = oracle.deconv2d_nhwc(x, w, 1, 2)
+    assert float(((y1 - yc).abs().double().cpu() / torch.as_tensor(b).clamp_min(1e-30)).max()) <= 1e-4
+
+
+def test_accuracy_band_paper_table3():
+    # PAPER.md Table 3 (lines 4125-4185): U[1,2] inputs, average relative error ~1e-7..1e-6 (Gamma8)
+    for r, tol_mean in ((3, 2e-6), (7, 2e-6), (9, 5e-5)):
+        y, yr, b = run_case("conv", 2, 16, 32, 64, 64, r, r, r // 2, r // 2, lo=1.0, hi=2.0)
+        assert_parity(y, yr, b)
+        rel = np.abs(y.cpu().double().numpy() - yr) / np.abs(yr)
+        assert rel.mean() < tol_mean, rel.mean()
