@@ -288,12 +288,13 @@ int run_fused(const Plan& pl, const float* x, const void* u, float* y, cudaStrea
 }
 
 int conv_common(int is_deconv, int N, int H, int W, int C, int K, int R, int S, int pad_h, int pad_w, const float* x,
-                const float* w, float* y, cudaStream_t stream, bool simt) {
+                const float* w, float* y, cudaStream_t stream, bool simt, unsigned long long* trace = nullptr) {
   if (!x || !w || !y) return I2CW_EINVAL;
   if (!aligned16(x) || !aligned16(w) || !aligned16(y)) return I2CW_EINVAL;
   Plan pl;
   int rc = make_plan(N, H, W, C, K, R, S, pad_h, pad_w, is_deconv, &pl);
   if (rc != I2CW_OK) return rc;
+  pl.trace = trace;
   if ((rc = bind_device_of(x)) != I2CW_OK) return rc;
   void* u = nullptr;
   const size_t ub = kUTagBytes + u_data_bytes(pl);
@@ -470,6 +471,14 @@ int i2cw_transform_matrices_rational(int m, int r, int point_set, int64_t* at_nu
 I2CW_API int i2cw_debug_conv_simt(int is_deconv, int N, int H, int W, int C, int K, int R, int S, int pad_h, int pad_w,
                          const float* x, const float* w, float* y, i2cw_stream_t stream) {
   return conv_common(is_deconv, N, H, W, C, K, R, S, pad_h, pad_w, x, w, y, (cudaStream_t)stream, true);
+}
+
+// Runs the product path with CTA 0's event timeline recorded into trace (device,
+// 16 kinds x 512 uint64 clock64 stamps; see trace_rec in common.cuh).
+I2CW_API int i2cw_debug_trace(int is_deconv, int N, int H, int W, int C, int K, int R, int S, int pad_h, int pad_w,
+                              const float* x, const float* w, float* y, unsigned long long* trace,
+                              i2cw_stream_t stream) {
+  return conv_common(is_deconv, N, H, W, C, K, R, S, pad_h, pad_w, x, w, y, (cudaStream_t)stream, false, trace);
 }
 
 I2CW_API int i2cw_debug_plan(int is_deconv, int N, int H, int W, int C, int K, int R, int S, int pad_h, int pad_w,

@@ -32,6 +32,7 @@ struct Plan {
   int GP, NPASS;        // points per pass (TMEM budget), passes = alpha / GP
   int NUS;              // U pipeline stages
   int smem_bytes;
+  unsigned long long* trace;  // debug timeline of CTA 0 (nullptr = off), see i2cw_debug_trace
   unsigned char lane_row[kMaxLanes];  // lane -> row within block (0xFF = idle lane)
   unsigned char lane_tw[kMaxLanes];   // lane -> tile within segment
 };
@@ -65,6 +66,10 @@ struct UTag {
 };
 
 #if defined(__CUDACC__)
+// Debug timeline: kind k, entry i -> trace[k * 512 + i] = clock64 (CTA 0 only).
+__device__ __forceinline__ void trace_rec(unsigned long long* tr, int kind, int i) {
+  if (tr != nullptr && blockIdx.x == 0 && i < 512) tr[kind * 512 + i] = clock64();
+}
 // ----------------------------------------------------------------------------
 // PTX helpers
 // ----------------------------------------------------------------------------

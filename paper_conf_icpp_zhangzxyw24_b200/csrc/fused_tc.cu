@@ -154,7 +154,9 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, GP, NWG>::NTHREADS, 1)
         for (int fh = 0; fh < pl.R; ++fh) {
           const int ks = cc * pl.R + fh;
           if (ks % NWG != g) continue;
+          if (l == 0) trace_rec(pl.trace, 3 * g + 0, vuse);
           if (vuse > 0) mbar_wait(&v_empty[g], (vuse - 1) & 1);
+          if (l == 0) trace_rec(pl.trace, 3 * g + 1, vuse);
           const int off = (has_slot ? (row_l + fh) : 0) * pl.WBOX + col0;
 #pragma unroll
           for (int h = 0; h < 2; ++h) {
@@ -201,12 +203,15 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, GP, NWG>::NTHREADS, 1)
           tmem_wait_st();
           tc_fence_before();
           mbar_arrive(&v_full[g]);
+          if (l == 0) trace_rec(pl.trace, 3 * g + 2, vuse);
           ++vuse;
         }
         mbar_arrive(&in_empty[st]);
       }
       // ---------------- epilogue of this pass: y (+)= A^T M ----------------
+      if (l == 0) trace_rec(pl.trace, 8 + g, 2 * PASS);
       mbar_wait(d_full, PASS & 1);
+      if (l == 0) trace_rec(pl.trace, 8 + g, 2 * PASS + 1);
       tc_fence_after();
       constexpr int CPW = NT / NWG;
 #pragma unroll 1
@@ -263,6 +268,7 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, GP, NWG>::NTHREADS, 1)
       }
       tc_fence_before();
       mbar_arrive(d_empty);
+      if (l == 0) trace_rec(pl.trace, 10 + g, PASS);
     });
   } else if (warp == NWG * 4) {
     // ============================ TMA producer ============================
@@ -306,11 +312,14 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, GP, NWG>::NTHREADS, 1)
         }
         for (int ks = 0; ks < pl.NKS; ++ks, ++ui) {
           const int g = ks % NWG;
+          trace_rec(pl.trace, 12, ui);
           mbar_wait(&v_full[g], vuse[g] & 1);
+          trace_rec(pl.trace, 13, ui);
           ++vuse[g];
           const int us = ui % NUS;
           mbar_wait(&u_full[us], (ui / NUS) & 1);
           tc_fence_after();
+          trace_rec(pl.trace, 6, ui);
           const uint32_t ub = u_base + us * UBYTES;
 #pragma unroll
           for (int tl = 0; tl < GP; ++tl) {
@@ -322,8 +331,10 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, GP, NWG>::NTHREADS, 1)
             mma_tf32_ts(dcol, a_hi, b_lo, idesc, 1u);
             mma_tf32_ts(dcol, a_hi, b_hi, idesc, 1u);
           }
+          trace_rec(pl.trace, 7, ui);
           mma_commit(&v_empty[g]);
           mma_commit(&u_empty[us]);
+          trace_rec(pl.trace, 14, ui);
         }
         mma_commit(d_full);
       }
