@@ -17,12 +17,13 @@
 namespace i2cw {
 cudaError_t launch_filter_transform(const float* w, float* u, int C, int K, int R, int S, int is_deconv, int alpha,
                                     int NT, int NB, int NCC, const double* G, cudaStream_t stream);
-cudaError_t launch_fused_tc(const CUtensorMap& xmap, const Plan& pl, const float* u, float* y, cudaStream_t stream);
+cudaError_t launch_fused_tc(const CUtensorMap& xmap, const CUtensorMap& ymap, const Plan& pl, const float* u,
+                            cudaStream_t stream);
 cudaError_t launch_fused_simt(const Plan& pl, const float* x, const float* u, float* y, cudaStream_t stream);
 
 namespace {
 
-constexpr int kNWG = 2;                // transform warpgroups in the tc kernel
+
 constexpr int kSmemBudget = 225 * 1024;
 
 // Per filter width S: F(m, S) and the point set. r = 2..7 follow the paper's
@@ -140,7 +141,9 @@ int make_plan(int N, int H, int W, int C, int K, int R, int S, int pad_h, int pa
   rows = std::min(rows, 256 - (R - 1));
   if (rows < 1) return I2CW_EUNSUPPORTED;
   const int ubytes = pl.GP * 2 * pl.NT * 32;
-  pl.NUS = 4;
+  const int NS = ns_for(pl.alpha, pl.NT);
+  pl.NUS = NS;
+  pl.NOB = 2;
   const int wmin = pl.TS * pl.m + S - 1;
   for (;;) {
     // balance rows over the row blocks of an image
@@ -158,11 +161,13 @@ int make_plan(int N, int H, int W, int C, int K, int R, int S, int pad_h, int pa
     pl.WBOX = bestw;
     pl.BOXB = pl.HBOX * pl.WBOX * 16;
     pl.PLANE = (pl.BOXB + 127) / 128 * 128;
-    const int bar_bytes = 8 * (2 * 2 + 2 * kNWG + 2 + 2 * pl.NUS) + 16;
-    pl.smem_bytes = pl.NUS * ubytes + 2 * 2 * pl.PLANE + bar_bytes;
+    pl.OSB = pl.ROWS * pl.TS * pl.m * 8 * 4;  // one 8-channel output slice of the CTA's rows
+    pl.OSTRIDE = (pl.OSB + 127) / 128 * 128;
+    const int bar_bytes = 8 * (2 * 2 + 2 * NS + 2) + 16;
+    pl.smem_bytes = NS * ubytes + 2 * 2 * pl.PLANE + kNWG * pl.NOB * pl.OSTRIDE + bar_bytes;
     if (pl.smem_bytes <= kSmemBudget) break;
-    if (pl.NUS > 2) { pl.NUS--; continue; }
-    if (rows > 1) { rows = rows / 2; continue; }
+    if (pl.NOB > 1) { pl.NOB = 1; continue; }
+    if (rows > 1) { rows = rows / 2; pl.NOB = 2; continue; }
     return I2CW_EUNSUPPORTED;
   }
   assign_lanes(pl.ROWS, pl.TS, pl.WBOX, pl.m, pl.lane_row, pl.lane_tw);
@@ -201,6 +206,20 @@ int encode_x_map(const Plan& pl, const float* x, CUtensorMap* map) {
   CUresult r = enc(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, const_cast<float*>(x), dims, strides, box, es,
                    CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS ? I2CW_OK : I2CW_EUNSUPPORTED;
+}
+
+// y: [N][P][Q][K] fp32; store box = 8 channels x TS*m columns x ROWS rows x 1 image
+// (elements outside [0,K) x [0,Q) x [0,P) are clipped by the TMA unit).
+int encode_y_map(const Plan& pl, float* y, CUtensorMap* map) {
+  PFN_encodeTiled_t enc = get_encode();
+  if (!enc) return I2CW_ECUDA;
+  cuuint64_t dims[4] = {(cuuint64_t)pl.K, (cuuint64_t)pl.Q, (cuuint64_t)pl.P, (cuuint64_t)pl.N};
+  cuuint64_t strides[3] = {(cuuint64_t)pl.K * 4, (cuuint64_t)pl.Q * pl.K * 4, (cuuint64_t)pl.P * pl.Q * pl.K * 4};
+  cuuint32_t box[4] = {8, (cuuint32_t)(pl.TS * pl.m), (cuuint32_t)pl.ROWS, 1};
+  cuuint32_t es[4] = {1, 1, 1, 1};
+  CUresult r = enc(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, y, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                   CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   return r == CUDA_SUCCESS ? I2CW_OK : I2CW_EUNSUPPORTED;
 }
 
@@ -280,11 +299,12 @@ int transform_into(const Plan& pl, int is_deconv, const float* w, void* u, cudaS
 }
 
 int run_fused(const Plan& pl, const float* x, const void* u, float* y, cudaStream_t stream) {
-  CUtensorMap map;
+  CUtensorMap map, ymap;
   int rc = encode_x_map(pl, x, &map);
   if (rc != I2CW_OK) return rc;
+  if ((rc = encode_y_map(pl, y, &ymap)) != I2CW_OK) return rc;
   const float* ud = reinterpret_cast<const float*>(static_cast<const uint8_t*>(u) + kUTagBytes);
-  return launch_fused_tc(map, pl, ud, y, stream) == cudaSuccess ? I2CW_OK : I2CW_ECUDA;
+  return launch_fused_tc(map, ymap, pl, ud, stream) == cudaSuccess ? I2CW_OK : I2CW_ECUDA;
 }
 
 int conv_common(int is_deconv, int N, int H, int W, int C, int K, int R, int S, int pad_h, int pad_w, const float* x,

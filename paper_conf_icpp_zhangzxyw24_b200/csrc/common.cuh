@@ -30,7 +30,10 @@ struct Plan {
   int PLANE;            // shared-memory stride between planes (BOXB rounded up to 128)
   int tile_blocks;      // N * PB * SEGS
   int GP, NPASS;        // points per pass (TMEM budget), passes = alpha / GP
-  int NUS;              // U pipeline stages
+  int NUS;              // U pipeline stages (v1 kernel; v2 uses the template NS)
+  int OSB;              // bytes of one output staging buffer = ROWS*TS*m*8*4 (TMA store box)
+  int OSTRIDE;          // OSB rounded up to 128
+  int NOB;              // output staging buffers per warpgroup (1 or 2)
   int smem_bytes;
   unsigned long long* trace;  // debug timeline of CTA 0 (nullptr = off), see i2cw_debug_trace
   unsigned char lane_row[kMaxLanes];  // lane -> row within block (0xFF = idle lane)
@@ -42,6 +45,18 @@ struct Plan {
 __host__ __device__ constexpr int gp_for(int alpha, int NT) {
   return NT == 64 ? 4 : (alpha % 8 == 0 ? 8 : 6);
 }
+// (U, V) k-step stages that fit next to the accumulators: NS * GP * 16 <= 512 - GP * NT,
+// capped at 4 and even (two transform warpgroups alternate stages).
+__host__ __device__ constexpr int ns_for(int alpha, int NT) {
+  return ((512 - gp_for(alpha, NT) * NT) / (gp_for(alpha, NT) * 16)) >= 4
+             ? 4
+             : (((512 - gp_for(alpha, NT) * NT) / (gp_for(alpha, NT) * 16)) / 2) * 2;
+}
+// MMA-issuing warps: one warp issues at most ~1 UMMA per 45 cycles (measured,
+// tools/mma_bench.cu), so several warps issue, each owning whole accumulators.
+__host__ __device__ constexpr int niss_for(int GP) { return GP % 4 == 0 ? 4 : (GP % 3 == 0 ? 3 : 2); }
+constexpr int kNWG = 2;  // transform / epilogue warpgroups
+__host__ __device__ constexpr int tc_threads(int GP) { return kNWG * 128 + 32 + niss_for(GP) * 32; }
 
 // Internal Winograd point order: singles {0, alpha-1} first, then the ± pairs
 // (1,2), (3,4), ... so that every pass of GP (even) points holds whole pairs
@@ -125,6 +140,37 @@ __device__ __forceinline__ void tma_load_4d(void* smem_dst, const CUtensorMap* m
       "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "r"(smem_u32(bar))
       : "memory");
 }
+// TMA: 4D tiled tensor store shared -> global (OOB elements of the box are not written)
+__device__ __forceinline__ void tma_store_4d(const CUtensorMap* map, const void* smem_src, int c0, int c1, int c2,
+                                             int c3) {
+  asm volatile("cp.async.bulk.tensor.4d.global.shared::cta.tile.bulk_group [%0, {%2, %3, %4, %5}], [%1];" ::"l"(
+                   reinterpret_cast<uint64_t>(map)),
+               "r"(smem_u32(smem_src)), "r"(c0), "r"(c1), "r"(c2), "r"(c3)
+               : "memory");
+}
+// TMA: 4D tiled reduce-add shared -> global (fp32 add performed at L2)
+__device__ __forceinline__ void tma_reduce_add_4d(const CUtensorMap* map, const void* smem_src, int c0, int c1,
+                                                  int c2, int c3) {
+  asm volatile(
+      "cp.reduce.async.bulk.tensor.4d.global.shared::cta.add.tile.bulk_group [%0, {%2, %3, %4, %5}], [%1];" ::"l"(
+          reinterpret_cast<uint64_t>(map)),
+      "r"(smem_u32(smem_src)), "r"(c0), "r"(c1), "r"(c2), "r"(c3)
+      : "memory");
+}
+__device__ __forceinline__ void bulk_commit_group() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void bulk_wait_group_read() {
+  asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory");
+}
+__device__ __forceinline__ void bulk_wait_group_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+// generic-proxy shared-memory writes -> visible to the async proxy (TMA store reads)
+__device__ __forceinline__ void fence_proxy_async_smem() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+__device__ __forceinline__ void named_bar_sync(int id, int nthreads) {
+  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
+}
+
 __device__ __forceinline__ void tma_prefetch_desc(const CUtensorMap* map) {
   asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(map)) : "memory");
 }
@@ -201,6 +247,13 @@ __device__ __forceinline__ float tf32_rna(float x) {
   uint32_t r;
   asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(r) : "f"(x));
   return __uint_as_float(r);
+}
+// 3xTF32 split on the ALU pipe: hi = x rounded to 10 mantissa bits (half away from
+// zero on the magnitude bits, == cvt.rna for finite x), lo = x - hi exactly in fp32
+// (the tensor core reads lo's top 19 bits; the dropped part is < 2^-21 |x|).
+__device__ __forceinline__ void split_tf32(float x, float& hi, float& lo) {
+  hi = __uint_as_float((__float_as_uint(x) + 0x1000u) & 0xFFFFE000u);
+  lo = x - hi;
 }
 
 // UMMA shared-memory descriptor, K-major, SWIZZLE_NONE (canonical interleaved

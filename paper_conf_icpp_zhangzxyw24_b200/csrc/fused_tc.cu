@@ -14,21 +14,26 @@
 //  * CTA = 128 Winograd tiles (UMMA M, one TMEM lane each) x NT output channels.
 //    Tiles are ROWS output rows x TS tiles of one image; lane->tile is a host
 //    permutation that spreads the 16-byte shared-memory reads over banks.
-//  * a2: one TMA warp stages, per 8-channel chunk, the (ROWS+R-1) x WBOX input
+//  * a2: a TMA warp stages, per 8-channel chunk, the (ROWS+R-1) x WBOX input
 //    rows of the block as two 16-byte channel planes (OOB zero fill = padding,
 //    PAPER.md:337-338); the rows are reused across all fh (vertical overlap)
 //    and by neighbouring windows (the (r-1) horizontal overlap, §5.4).
-//    U k-step images arrive by 1D bulk copy into a ring.
+//    The same warp streams each k-step's U image (1D bulk copy) into a ring.
 //  * a3: NWG transform warpgroups (thread = tile) read the alpha-window from
 //    shared memory, apply BT with zeros/±1 folded at compile time and the ±
 //    pair trick, split 3xTF32 hi/lo and write V into TMEM
-//    with tcgen05.st (V is the UMMA A operand, "TS" mode).
-//  * a4: one thread issues, per k-step and point, 3 tcgen05.mma.kind::tf32
-//    (lo*hi, hi*lo, hi*hi) into the point's fp32 accumulator in TMEM.
-//  * a5: after the last k-step the same warpgroups tcgen05.ld the accumulators,
-//    apply A^T in registers (pair trick) and store y with masked 16-byte stores.
-//  * TMEM budget: GP points x NT columns of accumulators + NWG V stages of
-//    GP x 16 columns <= 512; alpha/GP passes, pass > 0 adds into y (RMW).
+//    with tcgen05.st (V is the UMMA A operand, "TS" mode: no SMEM read for A).
+//  * a4: NISS issuer warps, each owning GP/NISS points' accumulators, issue per
+//    k-step 3 tcgen05.mma.kind::tf32 per point (lo*hi, hi*lo, hi*hi). Several
+//    issuers are needed: one warp issues at most one UMMA per ~45 cycles while
+//    a 128x64x8 tf32 UMMA takes 32 (tools/mma_bench.cu). Each accumulator has
+//    exactly one issuer, so results are bitwise deterministic.
+//  * k-step stages: NS slots, each = V (TMEM) + U (SMEM); one "full" barrier
+//    (128 transform arrivals + U tx bytes) and one "empty" barrier (NISS commits).
+//  * a5: the warpgroups tcgen05.ld the accumulators, apply A^T in registers
+//    (pair trick), stage 8-channel slices in shared memory and TMA-store them
+//    (TMA clips q >= Q, p >= P, k >= K: the in-kernel boundary). Passes > 0 use a
+//    TMA reduce-add into y (the accumulators hold GP of alpha points per pass).
 #include <utility>
 
 #include "common.cuh"
@@ -62,46 +67,52 @@ __device__ __forceinline__ float bt_dot(const float (&d)[A][4], int e) {
   return acc;
 }
 
-template <int M, int RW, int NT, int GP, int NWG>
+template <int M, int RW, int NT>
 struct TcCfg {
   using T = Wino<M, RW>;
   static constexpr int A = T::alpha;
+  static constexpr int GP = gp_for(A, NT);
+  static constexpr int NS = ns_for(A, NT);
+  static constexpr int NISS = niss_for(GP);
+  static constexpr int NWG = kNWG;
   static constexpr int NPASS = A / GP;
   static constexpr int NIS = 2;                       // input stages
   static constexpr int VCOL = GP * NT;                // first V column in TMEM
   static constexpr int TMEM_COLS = 512;
   static constexpr int UBYTES = GP * 2 * NT * 32;     // one k-step of U (GP points, hi+lo)
-  static constexpr int NTHREADS = NWG * 128 + 64;     // + TMA warp + MMA warp
+  static constexpr int NTHREADS = tc_threads(GP);
+  static constexpr int PPI = GP / NISS;               // points per issuer
   static_assert(A % GP == 0 && GP % 2 == 0, "passes must hold whole ± pairs");
-  static_assert(GP * NT + NWG * GP * 16 <= TMEM_COLS, "TMEM budget");
+  static_assert(NS >= 2 && NS % NWG == 0, "stage ring");
+  static_assert(GP * NT + NS * GP * 16 <= TMEM_COLS, "TMEM budget");
   static_assert(NT % 16 == 0 && NT >= 16 && NT <= 256, "UMMA N for M=128");
   static_assert((NT / NWG) % 8 == 0, "epilogue column split");
+  static_assert(GP % NISS == 0, "issuer split");
 };
 
-template <int M, int RW, int NT, int GP, int NWG>
-__global__ void __launch_bounds__(TcCfg<M, RW, NT, GP, NWG>::NTHREADS, 1)
-    fused_tc_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__ Plan pl,
-                    const float* __restrict__ u, float* __restrict__ y) {
-  using Cfg = TcCfg<M, RW, NT, GP, NWG>;
+template <int M, int RW, int NT>
+__global__ void __launch_bounds__(TcCfg<M, RW, NT>::NTHREADS, 1)
+    fused_tc_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__ CUtensorMap ymap,
+                    const __grid_constant__ Plan pl, const float* __restrict__ u) {
+  using Cfg = TcCfg<M, RW, NT>;
   using T = typename Cfg::T;
-  constexpr int A = Cfg::A, NPASS = Cfg::NPASS, NIS = Cfg::NIS, VCOL = Cfg::VCOL;
+  constexpr int A = Cfg::A, GP = Cfg::GP, NS = Cfg::NS, NISS = Cfg::NISS, NWG = Cfg::NWG;
+  constexpr int NPASS = Cfg::NPASS, NIS = Cfg::NIS, VCOL = Cfg::VCOL, PPI = Cfg::PPI;
   constexpr uint32_t UBYTES = Cfg::UBYTES;
 
   extern __shared__ __align__(1024) uint8_t smem[];
-  const int NUS = pl.NUS;
   const uint32_t inplane = (uint32_t)pl.PLANE;  // plane stride (128-aligned)
-  uint8_t* u_smem = smem;
-  uint8_t* in_smem = smem + (size_t)NUS * UBYTES;
-  uint64_t* bars = reinterpret_cast<uint64_t*>(in_smem + (size_t)NIS * 2 * inplane);
+  uint8_t* u_smem = smem;                                        // [NS][UBYTES]
+  uint8_t* in_smem = u_smem + (size_t)NS * UBYTES;               // [NIS][2 planes][PLANE]
+  uint8_t* o_smem = in_smem + (size_t)NIS * 2 * inplane;         // [NWG][NOB][OSTRIDE]
+  uint64_t* bars = reinterpret_cast<uint64_t*>(o_smem + (size_t)NWG * pl.NOB * pl.OSTRIDE);
   uint64_t* in_full = bars;             // [NIS]
   uint64_t* in_empty = in_full + NIS;   // [NIS]
-  uint64_t* v_full = in_empty + NIS;    // [NWG]
-  uint64_t* v_empty = v_full + NWG;     // [NWG]
-  uint64_t* d_full = v_empty + NWG;     // [1]
+  uint64_t* st_full = in_empty + NIS;   // [NS]
+  uint64_t* st_empty = st_full + NS;    // [NS]
+  uint64_t* d_full = st_empty + NS;     // [1]
   uint64_t* d_empty = d_full + 1;       // [1]
-  uint64_t* u_full = d_empty + 1;       // [NUS]
-  uint64_t* u_empty = u_full + NUS;     // [NUS]
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(u_empty + NUS);
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(d_empty + 1);
 
   const int warp = threadIdx.x / 32, lane32 = threadIdx.x % 32;
   const int b = blockIdx.x;
@@ -112,16 +123,16 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, GP, NWG>::NTHREADS, 1)
   const int rb = tb % pl.PB;
   const int n = tb / pl.PB;
   const int p0 = rb * pl.ROWS;
+  constexpr int PROD_WARP = NWG * 4, ISS_WARP0 = NWG * 4 + 1;
 
   if (threadIdx.x == 0) {
     for (int i = 0; i < NIS; ++i) { mbar_init(&in_full[i], 1); mbar_init(&in_empty[i], NWG * 128); }
-    for (int i = 0; i < NWG; ++i) { mbar_init(&v_full[i], 128); mbar_init(&v_empty[i], 1); }
-    mbar_init(d_full, 1);
+    for (int i = 0; i < NS; ++i) { mbar_init(&st_full[i], 128 + 1); mbar_init(&st_empty[i], NISS); }
+    mbar_init(d_full, NISS);
     mbar_init(d_empty, NWG * 128);
-    for (int i = 0; i < NUS; ++i) { mbar_init(&u_full[i], 1); mbar_init(&u_empty[i], 1); }
     fence_mbar_init();
   }
-  if (warp == NWG * 4 + 1) {  // MMA warp owns the TMEM allocation
+  if (warp == ISS_WARP0) {  // the first issuer warp owns the TMEM allocation
     tmem_alloc(tmem_slot, Cfg::TMEM_COLS);
     tmem_relinquish();
   }
@@ -129,6 +140,7 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, GP, NWG>::NTHREADS, 1)
   __syncthreads();
   tc_fence_after();
   const uint32_t tbase = *tmem_slot;
+  const int NKS = pl.NKS;
 
   if (warp < NWG * 4) {
     // ===================== transform + epilogue warpgroups =====================
@@ -136,27 +148,25 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, GP, NWG>::NTHREADS, 1)
     const int l = threadIdx.x % 128;  // TMEM lane == tile slot
     const int row_l = pl.lane_row[l], tw_l = pl.lane_tw[l];
     const bool has_slot = row_l != 0xFF;
-    const int p = p0 + (has_slot ? row_l : 0);
-    const int tw = seg * pl.TS + (has_slot ? tw_l : 0);
-    const bool valid = has_slot && p < pl.P && tw < pl.T_r;
-    const int q0 = tw * M;
     const int col0 = has_slot ? tw_l * M : 0;
     const uint32_t lane_addr = tbase + ((uint32_t)(l & ~31) << 16);
-    const uint32_t vbase = lane_addr + VCOL + g * GP * 16;
-    int vuse = 0;
+    const int TSM = pl.TS * M;  // output columns per CTA row segment
+    float* ostage = reinterpret_cast<float*>(o_smem + (size_t)g * pl.NOB * pl.OSTRIDE);
 
     static_for<NPASS>([&](auto PASS_) {
       constexpr int PASS = PASS_;
       for (int cc = 0; cc < pl.NCC; ++cc) {
-        const int li = PASS * pl.NCC + cc, st = li % NIS;
-        mbar_wait(&in_full[st], (li / NIS) & 1);
-        const float4* planes = reinterpret_cast<const float4*>(in_smem + (size_t)st * 2 * inplane);
+        const int li = PASS * pl.NCC + cc, ist = li % NIS;
+        mbar_wait(&in_full[ist], (li / NIS) & 1);
+        const float4* planes = reinterpret_cast<const float4*>(in_smem + (size_t)ist * 2 * inplane);
         for (int fh = 0; fh < pl.R; ++fh) {
-          const int ks = cc * pl.R + fh;
-          if (ks % NWG != g) continue;
-          if (l == 0) trace_rec(pl.trace, 3 * g + 0, vuse);
-          if (vuse > 0) mbar_wait(&v_empty[g], (vuse - 1) & 1);
-          if (l == 0) trace_rec(pl.trace, 3 * g + 1, vuse);
+          const int kg = PASS * NKS + cc * pl.R + fh;  // global k-step index
+          if (kg % NWG != g) continue;
+          const int s = kg % NS, use = kg / NS;
+          if (l == 0) trace_rec(pl.trace, 3 * g + 0, kg / NWG);
+          if (use > 0) mbar_wait(&st_empty[s], (use - 1) & 1);
+          if (l == 0) trace_rec(pl.trace, 3 * g + 1, kg / NWG);
+          const uint32_t vbase = lane_addr + VCOL + s * GP * 16;
           const int off = (has_slot ? (row_l + fh) : 0) * pl.WBOX + col0;
 #pragma unroll
           for (int h = 0; h < 2; ++h) {
@@ -190,8 +200,8 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, GP, NWG>::NTHREADS, 1)
               float ha[4], la[4], hb[4], lb[4];
 #pragma unroll
               for (int e = 0; e < 4; ++e) {
-                ha[e] = tf32_rna(va[e]); la[e] = tf32_rna(va[e] - ha[e]);
-                hb[e] = tf32_rna(vb[e]); lb[e] = tf32_rna(vb[e] - hb[e]);
+                split_tf32(va[e], ha[e], la[e]);
+                split_tf32(vb[e], hb[e], lb[e]);
               }
               const uint32_t ca = vbase + tl0 * 16 + h * 4, cb = ca + 16;
               tmem_st_x4(ca, ha[0], ha[1], ha[2], ha[3]);
@@ -202,18 +212,18 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, GP, NWG>::NTHREADS, 1)
           }
           tmem_wait_st();
           tc_fence_before();
-          mbar_arrive(&v_full[g]);
-          if (l == 0) trace_rec(pl.trace, 3 * g + 2, vuse);
-          ++vuse;
+          mbar_arrive(&st_full[s]);
+          if (l == 0) trace_rec(pl.trace, 3 * g + 2, kg / NWG);
         }
-        mbar_arrive(&in_empty[st]);
+        mbar_arrive(&in_empty[ist]);
       }
-      // ---------------- epilogue of this pass: y (+)= A^T M ----------------
+      // ---------- epilogue of this pass: y (+)= A^T M via shared memory + TMA ----------
       if (l == 0) trace_rec(pl.trace, 8 + g, 2 * PASS);
       mbar_wait(d_full, PASS & 1);
-      if (l == 0) trace_rec(pl.trace, 8 + g, 2 * PASS + 1);
       tc_fence_after();
+      if (l == 0) trace_rec(pl.trace, 8 + g, 2 * PASS + 1);
       constexpr int CPW = NT / NWG;
+      const int qbase = seg * TSM;
 #pragma unroll 1
       for (int c8 = 0; c8 < CPW / 8; ++c8) {
         const int col = g * CPW + c8 * 8;
@@ -221,8 +231,18 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, GP, NWG>::NTHREADS, 1)
 #pragma unroll
         for (int tl = 0; tl < GP; ++tl) tmem_ld_x8(lane_addr + tl * NT + col, Mt[tl]);
         tmem_wait_ld();
-        // pair sums / differences (internal slots 2q, 2q+1 hold points a, a+1)
-        const int k0 = nb * NT + col;
+        if (c8 == CPW / 8 - 1) {  // accumulators fully read: the issuers may start the next pass
+          tc_fence_before();
+          mbar_arrive(d_empty);
+        }
+        // staging buffer reuse: the TMA store that last read it must be done reading
+        const int ob = pl.NOB == 2 ? (c8 & 1) : 0;
+        if (l == 0) {
+          if (pl.NOB == 2) bulk_wait_group_read<1>();
+          else bulk_wait_group_read<0>();
+        }
+        named_bar_sync(1 + g, 128);
+        float* stg = ostage + (size_t)ob * (pl.OSTRIDE / 4);
         static_for<M>([&](auto I_) {
           constexpr int i = I_;
           float o[8];
@@ -243,98 +263,92 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, GP, NWG>::NTHREADS, 1)
               constexpr float ca = T::AT(i, pa);
 #pragma unroll
               for (int e = 0; e < 8; ++e) {
-                const float s = (i % 2 == 0) ? (Mt[tl0][e] + Mt[tl0 + 1][e]) : (Mt[tl0][e] - Mt[tl0 + 1][e]);
-                if constexpr (ca == 1.f) o[e] += s;
-                else if constexpr (ca != 0.f) o[e] = fmaf(ca, s, o[e]);
+                const float sv = (i % 2 == 0) ? (Mt[tl0][e] + Mt[tl0 + 1][e]) : (Mt[tl0][e] - Mt[tl0 + 1][e]);
+                if constexpr (ca == 1.f) o[e] += sv;
+                else if constexpr (ca != 0.f) o[e] = fmaf(ca, sv, o[e]);
               }
             }
           });
-          if (valid && q0 + i < pl.Q) {
-            float* yp = y + (((size_t)n * pl.P + p) * pl.Q + q0 + i) * pl.K + k0;
-#pragma unroll
-            for (int hh = 0; hh < 2; ++hh) {
-              if (k0 + hh * 4 + 4 <= pl.K) {
-                float4 v = make_float4(o[hh * 4 + 0], o[hh * 4 + 1], o[hh * 4 + 2], o[hh * 4 + 3]);
-                float4* dst = reinterpret_cast<float4*>(yp + hh * 4);
-                if constexpr (PASS > 0) {
-                  const float4 prev = *dst;
-                  v.x += prev.x; v.y += prev.y; v.z += prev.z; v.w += prev.w;
-                }
-                *dst = v;
-              }
-            }
+          if (has_slot) {
+            float4* dst = reinterpret_cast<float4*>(stg + ((size_t)row_l * TSM + tw_l * M + i) * 8);
+            dst[0] = make_float4(o[0], o[1], o[2], o[3]);
+            dst[1] = make_float4(o[4], o[5], o[6], o[7]);
           }
         });
+        fence_proxy_async_smem();
+        named_bar_sync(1 + g, 128);
+        if (l == 0) {
+          const int k0 = nb * NT + col;
+          if constexpr (PASS == 0) tma_store_4d(&ymap, stg, k0, qbase, p0, n);
+          else tma_reduce_add_4d(&ymap, stg, k0, qbase, p0, n);
+          bulk_commit_group();
+        }
       }
-      tc_fence_before();
-      mbar_arrive(d_empty);
+      // this pass's writes must be complete before the next pass's reduce-add
+      if (l == 0) bulk_wait_group_all();
       if (l == 0) trace_rec(pl.trace, 10 + g, PASS);
     });
-  } else if (warp == NWG * 4) {
-    // ============================ TMA producer ============================
+  } else if (warp == PROD_WARP) {
+    // ====================== TMA / bulk-copy producer ======================
     if (lane32 == 0) {
       tma_prefetch_desc(&xmap);
+      tma_prefetch_desc(&ymap);
       const int wstart = seg * pl.TS * M - pl.pad_w;
       const int hstart = p0 - pl.pad_h;
-      int ui = 0;
       for (int pass = 0; pass < NPASS; ++pass) {
         for (int cc = 0; cc < pl.NCC; ++cc) {
-          const int li = pass * pl.NCC + cc, st = li % NIS;
-          if (li >= NIS) mbar_wait(&in_empty[st], ((li / NIS) - 1) & 1);
-          uint8_t* dst = in_smem + (size_t)st * 2 * inplane;
-          mbar_expect_tx(&in_full[st], 2u * (uint32_t)pl.BOXB);
-          tma_load_4d(dst, &xmap, &in_full[st], cc * 8, wstart, hstart, n);
-          tma_load_4d(dst + inplane, &xmap, &in_full[st], cc * 8 + 4, wstart, hstart, n);
-          for (int fh = 0; fh < pl.R; ++fh, ++ui) {
-            const int ks = cc * pl.R + fh, us = ui % NUS;
-            if (ui >= NUS) mbar_wait(&u_empty[us], ((ui / NUS) - 1) & 1);
-            mbar_expect_tx(&u_full[us], UBYTES);
-            bulk_load(u_smem + (size_t)us * UBYTES, u + u_offset(NT, A, nb, pl.NKS, ks, pass * GP, 0), UBYTES,
-                      &u_full[us]);
+          const int li = pass * pl.NCC + cc, ist = li % NIS;
+          if (li >= NIS) mbar_wait(&in_empty[ist], ((li / NIS) - 1) & 1);
+          uint8_t* dst = in_smem + (size_t)ist * 2 * inplane;
+          mbar_expect_tx(&in_full[ist], 2u * (uint32_t)pl.BOXB);
+          tma_load_4d(dst, &xmap, &in_full[ist], cc * 8, wstart, hstart, n);
+          tma_load_4d(dst + inplane, &xmap, &in_full[ist], cc * 8 + 4, wstart, hstart, n);
+          for (int fh = 0; fh < pl.R; ++fh) {
+            const int ks = cc * pl.R + fh, kg = pass * NKS + ks;
+            const int s = kg % NS, use = kg / NS;
+            if (use > 0) mbar_wait(&st_empty[s], (use - 1) & 1);
+            mbar_expect_tx(&st_full[s], UBYTES);
+            bulk_load(u_smem + (size_t)s * UBYTES, u + u_offset(NT, A, nb, NKS, ks, pass * GP, 0), UBYTES,
+                      &st_full[s]);
           }
         }
       }
     }
     __syncwarp();
   } else {
-    // ============================= MMA issuer =============================
+    // ============================= MMA issuers =============================
+    const int iss = warp - ISS_WARP0;  // owns points tl = iss * PPI .. iss * PPI + PPI - 1
     if (lane32 == 0) {
       constexpr uint32_t idesc = idesc_tf32(128, NT);
       const uint32_t u_base = smem_u32(u_smem);
-      int ui = 0;
-      int vuse[NWG];
-#pragma unroll
-      for (int i = 0; i < NWG; ++i) vuse[i] = 0;
       for (int pass = 0; pass < NPASS; ++pass) {
         if (pass > 0) {
           mbar_wait(d_empty, (pass - 1) & 1);
           tc_fence_after();
         }
-        for (int ks = 0; ks < pl.NKS; ++ks, ++ui) {
-          const int g = ks % NWG;
-          trace_rec(pl.trace, 12, ui);
-          mbar_wait(&v_full[g], vuse[g] & 1);
-          trace_rec(pl.trace, 13, ui);
-          ++vuse[g];
-          const int us = ui % NUS;
-          mbar_wait(&u_full[us], (ui / NUS) & 1);
+        for (int ks = 0; ks < NKS; ++ks) {
+          const int kg = pass * NKS + ks;
+          const int s = kg % NS, use = kg / NS;
+          if (iss == 0) trace_rec(pl.trace, 12, kg);
+          mbar_wait(&st_full[s], use & 1);
           tc_fence_after();
-          trace_rec(pl.trace, 6, ui);
-          const uint32_t ub = u_base + us * UBYTES;
+          if (iss == 0) trace_rec(pl.trace, 6, kg);
+          const uint32_t ub = u_base + s * UBYTES;
+          const uint32_t va = tbase + VCOL + s * GP * 16;
+          // product order lo*hi, hi*lo, hi*hi (small terms first), points innermost
 #pragma unroll
-          for (int tl = 0; tl < GP; ++tl) {
-            const uint32_t a_hi = tbase + VCOL + g * GP * 16 + tl * 16, a_lo = a_hi + 8;
-            const uint64_t b_hi = umma_desc_kmajor_noswizzle(ub + (tl * 2 + 0) * NT * 32, NT * 16, 128);
-            const uint64_t b_lo = umma_desc_kmajor_noswizzle(ub + (tl * 2 + 1) * NT * 32, NT * 16, 128);
-            const uint32_t dcol = tbase + tl * NT;
-            mma_tf32_ts(dcol, a_lo, b_hi, idesc, ks > 0 ? 1u : 0u);
-            mma_tf32_ts(dcol, a_hi, b_lo, idesc, 1u);
-            mma_tf32_ts(dcol, a_hi, b_hi, idesc, 1u);
+          for (int prod = 0; prod < 3; ++prod) {
+#pragma unroll
+            for (int pi = 0; pi < PPI; ++pi) {
+              const int tl = iss * PPI + pi;
+              const uint32_t a = va + tl * 16 + (prod == 0 ? 8 : 0);
+              const uint64_t bd = umma_desc_kmajor_noswizzle(ub + (tl * 2 + (prod == 1 ? 1 : 0)) * NT * 32, NT * 16, 128);
+              mma_tf32_ts(tbase + tl * NT, a, bd, idesc, (ks > 0 || prod > 0) ? 1u : 0u);
+            }
           }
-          trace_rec(pl.trace, 7, ui);
-          mma_commit(&v_empty[g]);
-          mma_commit(&u_empty[us]);
-          trace_rec(pl.trace, 14, ui);
+          if (iss == 0) trace_rec(pl.trace, 7, kg);
+          mma_commit(&st_empty[s]);
+          if (iss == 0) trace_rec(pl.trace, 14, kg);
         }
         mma_commit(d_full);
       }
@@ -344,32 +358,31 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, GP, NWG>::NTHREADS, 1)
 
   tc_fence_before();
   __syncthreads();
-  if (warp == NWG * 4 + 1) {
+  if (warp == ISS_WARP0) {
     tc_fence_after();
     tmem_dealloc(tbase, Cfg::TMEM_COLS);
   }
 }
 
-template <int M, int RW, int NT, int GP>
-static cudaError_t launch_tc_t(const CUtensorMap& xmap, const Plan& pl, const float* u, float* y,
+template <int M, int RW, int NT>
+static cudaError_t launch_tc_t(const CUtensorMap& xmap, const CUtensorMap& ymap, const Plan& pl, const float* u,
                                cudaStream_t stream) {
-  constexpr int NWG = 2;
-  using Cfg = TcCfg<M, RW, NT, GP, NWG>;
-  auto kern = fused_tc_kernel<M, RW, NT, GP, NWG>;
+  using Cfg = TcCfg<M, RW, NT>;
+  auto kern = fused_tc_kernel<M, RW, NT>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, pl.smem_bytes);
   if (e != cudaSuccess) return e;
-  kern<<<pl.tile_blocks * pl.NB, Cfg::NTHREADS, pl.smem_bytes, stream>>>(xmap, pl, u, y);
+  kern<<<pl.tile_blocks * pl.NB, Cfg::NTHREADS, pl.smem_bytes, stream>>>(xmap, ymap, pl, u);
   return cudaGetLastError();
 }
 
-// (m, r) -> kernel instantiation for the two N tiles; GP from the TMEM budget
-// (NT=64: GP=4; NT=32: GP=8), see make_plan() in api.cu.
-cudaError_t launch_fused_tc(const CUtensorMap& xmap, const Plan& pl, const float* u, float* y, cudaStream_t stream) {
+// (m, r, NT) -> kernel instantiation (GP, NS, NISS derived; see common.cuh).
+cudaError_t launch_fused_tc(const CUtensorMap& xmap, const CUtensorMap& ymap, const Plan& pl, const float* u,
+                            cudaStream_t stream) {
   const int key = pl.S * 1000 + pl.m * 10 + (pl.NT == 64 ? 1 : 0);
   switch (key) {
-#define I2CW_TC(MM, RR)                                                                               \
-  case RR * 1000 + MM * 10 + 1: return launch_tc_t<MM, RR, 64, gp_for(MM + RR - 1, 64)>(xmap, pl, u, y, stream); \
-  case RR * 1000 + MM * 10 + 0: return launch_tc_t<MM, RR, 32, gp_for(MM + RR - 1, 32)>(xmap, pl, u, y, stream);
+#define I2CW_TC(MM, RR)                                                                          \
+  case RR * 1000 + MM * 10 + 1: return launch_tc_t<MM, RR, 64>(xmap, ymap, pl, u, stream); \
+  case RR * 1000 + MM * 10 + 0: return launch_tc_t<MM, RR, 32>(xmap, ymap, pl, u, stream);
     I2CW_TC(7, 2) I2CW_TC(6, 3) I2CW_TC(5, 4) I2CW_TC(4, 5) I2CW_TC(3, 6) I2CW_TC(2, 7)  // alpha 8
     I2CW_TC(5, 8) I2CW_TC(4, 9)                                                          // alpha 12
     I2CW_TC(10, 7) I2CW_TC(9, 8) I2CW_TC(8, 9)                                           // alpha 16 (ablation)

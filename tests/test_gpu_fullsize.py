@@ -21,8 +21,8 @@ FULL = [("conv", 128, 56, 56, 64, 64, 3, 3, 1, 1)] + \
 def test_full_size_sampled(cfg):
     kind, N, H, W, C, K, R, S, ph, pw = cfg
     g = torch.Generator(device="cuda").manual_seed(1234)
-    x = (torch.rand((N, H, W, C), generator=g, device="cuda") * 2 - 1).contiguous()
-    w = (torch.rand((K, R, S, C) if kind == "conv" else (C, R, S, K), generator=g, device="cuda") * 2 - 1).contiguous()
+    x = (torch.rand((N, H, W, C), generator=g, device="cuda", dtype=torch.float32) * 2 - 1).contiguous()
+    w = (torch.rand((K, R, S, C) if kind == "conv" else (C, R, S, K), generator=g, device="cuda", dtype=torch.float32) * 2 - 1).contiguous()
     y = (i2cw.conv2d_nhwc if kind == "conv" else i2cw.deconv2d_nhwc)(x, w, ph, pw)
     torch.cuda.synchronize()
     assert bool(torch.isfinite(y).all())

