@@ -54,49 +54,44 @@ bool choose(int S, Choice* c) {
 
 inline int cdiv(int a, int b) { return (a + b - 1) / b; }
 
-// lane -> (row, tile) permutation: every 8 consecutive lanes (one LDS.128
-// quarter-warp wavefront) should start at distinct 16-byte bank groups,
-// i.e. distinct (row * WBOX + tw * m) mod 8. Greedy over residue buckets.
-// Returns the summed conflict degree (0 = conflict-free).
-int assign_lanes(int ROWS, int TS, int WBOX, int m, unsigned char* lrow, unsigned char* ltw) {
-  std::vector<std::pair<int, int>> bucket[8];
+// lane -> (row, tile) permutation. Every 8 consecutive lanes form one quarter-warp
+// shared-memory wavefront for two access patterns:
+//  * input reads (LDS.128 of 16-byte columns): bank group (row*WBOX + tw*m) mod 8;
+//  * staged output writes (swizzled 128B/64B rows r = row*TS + tw): r & 7, or (r>>1) & 3.
+// Greedy: fill each group with the tile adding the fewest repeated residues.
+// Returns the summed conflict degree (0 = both conflict-free).
+int assign_lanes(int ROWS, int TS, int WBOX, int m, int cpw, unsigned char* lrow, unsigned char* ltw) {
+  struct Tile { int r, t, in, out; };
+  std::vector<Tile> pool;
   for (int r = 0; r < ROWS; ++r)
-    for (int t = 0; t < TS; ++t) bucket[(r * WBOX + t * m) % 8].push_back({r, t});
+    for (int t = 0; t < TS; ++t) {
+      const int orow = r * TS + t;
+      pool.push_back({r, t, (r * WBOX + t * m) % 8, cpw == 32 ? (orow & 7) : ((orow >> 1) & 3)});
+    }
   std::fill(lrow, lrow + kMaxLanes, 0xFF);
   std::fill(ltw, ltw + kMaxLanes, 0);
   int lane = 0, cost = 0;
-  const int total = ROWS * TS;
-  while (lane < total) {
-    int cnt[8] = {0};
-    int in_group = 0;
-    // first pass: distinct residues, fullest buckets first
-    int order[8];
-    for (int i = 0; i < 8; ++i) order[i] = i;
-    std::sort(order, order + 8, [&](int a, int b) { return bucket[a].size() > bucket[b].size(); });
-    for (int oi = 0; oi < 8 && in_group < 8 && lane < total; ++oi) {
-      auto& bk = bucket[order[oi]];
-      if (bk.empty()) continue;
-      lrow[lane] = (unsigned char)bk.back().first;
-      ltw[lane] = (unsigned char)bk.back().second;
-      bk.pop_back();
-      cnt[order[oi]]++;
-      ++lane; ++in_group;
+  std::vector<char> used(pool.size(), 0);
+  while (lane < (int)pool.size()) {
+    int cin[8] = {0}, cout_[8] = {0};
+    for (int k = 0; k < 8 && lane < (int)pool.size(); ++k) {
+      int best = -1, bestc = 1 << 30;
+      for (size_t i = 0; i < pool.size(); ++i) {
+        if (used[i]) continue;
+        const int c = 2 * cin[pool[i].in] + cout_[pool[i].out];
+        if (c < bestc) { bestc = c; best = (int)i; }
+        if (c == 0) break;
+      }
+      used[best] = 1;
+      cin[pool[best].in]++;
+      cout_[pool[best].out]++;
+      lrow[lane] = (unsigned char)pool[best].r;
+      ltw[lane] = (unsigned char)pool[best].t;
+      ++lane;
     }
-    // fill the rest of the group (conflicting)
-    while (in_group < 8 && lane < total) {
-      int best = -1;
-      for (int i = 0; i < 8; ++i)
-        if (!bucket[i].empty() && (best < 0 || bucket[i].size() > bucket[best].size())) best = i;
-      auto& bk = bucket[best];
-      lrow[lane] = (unsigned char)bk.back().first;
-      ltw[lane] = (unsigned char)bk.back().second;
-      bk.pop_back();
-      cnt[best]++;
-      ++lane; ++in_group;
-    }
-    int mx = 0;
-    for (int i = 0; i < 8; ++i) mx = std::max(mx, cnt[i]);
-    cost += mx - 1;
+    int mi = 0, mo = 0;
+    for (int i = 0; i < 8; ++i) { mi = std::max(mi, cin[i]); mo = std::max(mo, cout_[i]); }
+    cost += (mi - 1) + (cpw == 32 ? (mo - 1) : std::max(0, mo - 2));
   }
   return cost;
 }
@@ -144,6 +139,7 @@ int make_plan(int N, int H, int W, int C, int K, int R, int S, int pad_h, int pa
   const int NS = ns_for(pl.alpha, pl.NT);
   pl.NUS = NS;
   pl.NOB = 2;
+  pl.NIS = 4;
   const int wmin = pl.TS * pl.m + S - 1;
   for (;;) {
     // balance rows over the row blocks of an image
@@ -155,22 +151,37 @@ int make_plan(int N, int H, int W, int C, int K, int R, int S, int pad_h, int pa
     int best = -1, bestw = wmin;
     for (int wb = wmin; wb <= std::min(256, wmin + 7); ++wb) {
       unsigned char lr[kMaxLanes], lt[kMaxLanes];
-      const int c = assign_lanes(pl.ROWS, pl.TS, wb, pl.m, lr, lt);
+      const int c = assign_lanes(pl.ROWS, pl.TS, wb, pl.m, pl.NT / nwg_for(pl.NT), lr, lt);
       if (best < 0 || c < best) { best = c; bestw = wb; }
     }
     pl.WBOX = bestw;
     pl.BOXB = pl.HBOX * pl.WBOX * 16;
     pl.PLANE = (pl.BOXB + 127) / 128 * 128;
-    pl.OSB = pl.ROWS * pl.TS * pl.m * 8 * 4;  // one 8-channel output slice of the CTA's rows
-    pl.OSTRIDE = (pl.OSB + 127) / 128 * 128;
-    const int bar_bytes = 8 * (2 * 2 + 2 * NS + 2) + 16;
-    pl.smem_bytes = NS * ubytes + 2 * 2 * pl.PLANE + kNWG * pl.NOB * pl.OSTRIDE + bar_bytes;
-    if (pl.smem_bytes <= kSmemBudget) break;
-    if (pl.NOB > 1) { pl.NOB = 1; continue; }
-    if (rows > 1) { rows = rows / 2; pl.NOB = 2; continue; }
+    // Output staging: one output column i of every tile, NT/2 channels per warpgroup
+    // (one 128- or 64-byte swizzled row per tile), stored by TMA with Q stride m.
+    pl.OPITCH = pl.TS * pl.m;
+    pl.OSB = pl.ROWS * pl.TS * (pl.NT / nwg_for(pl.NT)) * 4;
+    pl.OSTRIDE = (pl.OSB + 1023) / 1024 * 1024;
+    // ring depths, most preferred first: U slots hide the L2 latency of the filter
+    // stream (~1-2K cycles), input stages that of the row boxes, 2 output buffers
+    // overlap the TMA store of one output column with the next.
+    static const int kDepths[][3] = {{8, 3, 2}, {8, 3, 1}, {6, 3, 2}, {6, 3, 1}, {6, 2, 1},
+                                     {4, 3, 1}, {4, 2, 1}, {3, 2, 1}, {2, 2, 1}};
+    bool fit = false;
+    for (const auto& d : kDepths) {
+      pl.NUS = std::max(d[0], NS);
+      pl.NIS = d[1];
+      pl.NOB = d[2];
+      const int bar_bytes = 8 * (2 * pl.NIS + 2 * NS + 2 + 2 * pl.NUS) + 16;
+      pl.smem_bytes =
+          pl.NUS * ubytes + pl.NIS * 2 * pl.PLANE + nwg_for(pl.NT) * pl.NOB * pl.OSTRIDE + bar_bytes;
+      if (pl.smem_bytes <= kSmemBudget) { fit = true; break; }
+    }
+    if (fit) break;
+    if (rows > 1) { rows = rows / 2; continue; }
     return I2CW_EUNSUPPORTED;
   }
-  assign_lanes(pl.ROWS, pl.TS, pl.WBOX, pl.m, pl.lane_row, pl.lane_tw);
+  assign_lanes(pl.ROWS, pl.TS, pl.WBOX, pl.m, pl.NT / nwg_for(pl.NT), pl.lane_row, pl.lane_tw);
   pl.tile_blocks = N * pl.PB * pl.SEGS;
   *out = pl;
   return I2CW_OK;
@@ -209,17 +220,20 @@ int encode_x_map(const Plan& pl, const float* x, CUtensorMap* map) {
   return r == CUDA_SUCCESS ? I2CW_OK : I2CW_EUNSUPPORTED;
 }
 
-// y: [N][P][Q][K] fp32; store box = 8 channels x TS*m columns x ROWS rows x 1 image
-// (elements outside [0,K) x [0,Q) x [0,P) are clipped by the TMA unit).
+// y: [N][P][Q][K] fp32; store box = NT/2 channels x (TS*m columns walked with element
+// stride m, i.e. TS positions q0 + i) x ROWS rows x 1 image, 128B/64B swizzled.
+// Elements outside [0,K) x [0,Q) x [0,P) are clipped by the TMA unit (the in-kernel boundary).
 int encode_y_map(const Plan& pl, float* y, CUtensorMap* map) {
   PFN_encodeTiled_t enc = get_encode();
   if (!enc) return I2CW_ECUDA;
+  const int cpw = pl.NT / nwg_for(pl.NT);
   cuuint64_t dims[4] = {(cuuint64_t)pl.K, (cuuint64_t)pl.Q, (cuuint64_t)pl.P, (cuuint64_t)pl.N};
   cuuint64_t strides[3] = {(cuuint64_t)pl.K * 4, (cuuint64_t)pl.Q * pl.K * 4, (cuuint64_t)pl.P * pl.Q * pl.K * 4};
-  cuuint32_t box[4] = {8, (cuuint32_t)(pl.TS * pl.m), (cuuint32_t)pl.ROWS, 1};
-  cuuint32_t es[4] = {1, 1, 1, 1};
+  cuuint32_t box[4] = {(cuuint32_t)cpw, (cuuint32_t)(pl.TS * pl.m), (cuuint32_t)pl.ROWS, 1};
+  cuuint32_t es[4] = {1, (cuuint32_t)pl.m, 1, 1};
   CUresult r = enc(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, y, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                   CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+                   cpw == 32 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B,
+                   CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   return r == CUDA_SUCCESS ? I2CW_OK : I2CW_EUNSUPPORTED;
 }
 
@@ -494,7 +508,7 @@ I2CW_API int i2cw_debug_conv_simt(int is_deconv, int N, int H, int W, int C, int
 }
 
 // Runs the product path with CTA 0's event timeline recorded into trace (device,
-// 16 kinds x 512 uint64 clock64 stamps; see trace_rec in common.cuh).
+// 32 kinds x 512 uint64 clock64 stamps; see trace_rec in common.cuh).
 I2CW_API int i2cw_debug_trace(int is_deconv, int N, int H, int W, int C, int K, int R, int S, int pad_h, int pad_w,
                               const float* x, const float* w, float* y, unsigned long long* trace,
                               i2cw_stream_t stream) {

@@ -31,9 +31,11 @@ struct Plan {
   int tile_blocks;      // N * PB * SEGS
   int GP, NPASS;        // points per pass (TMEM budget), passes = alpha / GP
   int NUS;              // U pipeline stages (v1 kernel; v2 uses the template NS)
-  int OSB;              // bytes of one output staging buffer = ROWS*TS*m*8*4 (TMA store box)
-  int OSTRIDE;          // OSB rounded up to 128
+  int OPITCH;           // (unused, kept for the debug plan layout)
+  int OSB;              // bytes of one output staging buffer = ROWS*TS*(NT/2)*4 (TMA store box)
+  int OSTRIDE;          // OSB rounded up to 1024 (swizzled TMA boxes need 1024-byte alignment)
   int NOB;              // output staging buffers per warpgroup (1 or 2)
+  int NIS;              // input (x row box) stages
   int smem_bytes;
   unsigned long long* trace;  // debug timeline of CTA 0 (nullptr = off), see i2cw_debug_trace
   unsigned char lane_row[kMaxLanes];  // lane -> row within block (0xFF = idle lane)
@@ -55,8 +57,11 @@ __host__ __device__ constexpr int ns_for(int alpha, int NT) {
 // MMA-issuing warps: one warp issues at most ~1 UMMA per 45 cycles (measured,
 // tools/mma_bench.cu), so several warps issue, each owning whole accumulators.
 __host__ __device__ constexpr int niss_for(int GP) { return GP % 4 == 0 ? 4 : (GP % 3 == 0 ? 3 : 2); }
-constexpr int kNWG = 2;  // transform / epilogue warpgroups
-__host__ __device__ constexpr int tc_threads(int GP) { return kNWG * 128 + 32 + niss_for(GP) * 32; }
+// Transform / epilogue warpgroups: the input transform of one k-step by one
+// warpgroup (one warp per SMSP) is latency-bound, so NT=64 (4 stages) uses 4
+// warpgroups, each owning one stage and 16 output channels in the epilogue.
+__host__ __device__ constexpr int nwg_for(int NT) { return NT == 64 ? 4 : 2; }
+__host__ __device__ constexpr int tc_threads(int GP, int NT) { return nwg_for(NT) * 128 + 64 + niss_for(GP) * 32; }
 
 // Internal Winograd point order: singles {0, alpha-1} first, then the ± pairs
 // (1,2), (3,4), ... so that every pass of GP (even) points holds whole pairs
@@ -239,6 +244,18 @@ __device__ __forceinline__ void tmem_ld_x8(uint32_t taddr, float* v) {
                : "memory");
 #pragma unroll
   for (int i = 0; i < 8; ++i) v[i] = __uint_as_float(r[i]);
+}
+__device__ __forceinline__ void tmem_ld_x16(uint32_t taddr, float* v) {
+  uint32_t r[16];
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, "
+      "%15}, [%16];"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]), "=r"(r[8]),
+        "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
+      : "r"(taddr)
+      : "memory");
+#pragma unroll
+  for (int i = 0; i < 16; ++i) v[i] = __uint_as_float(r[i]);
 }
 __device__ __forceinline__ void tmem_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
 

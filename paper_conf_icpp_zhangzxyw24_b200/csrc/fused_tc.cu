@@ -74,13 +74,12 @@ struct TcCfg {
   static constexpr int GP = gp_for(A, NT);
   static constexpr int NS = ns_for(A, NT);
   static constexpr int NISS = niss_for(GP);
-  static constexpr int NWG = kNWG;
+  static constexpr int NWG = nwg_for(NT);
   static constexpr int NPASS = A / GP;
-  static constexpr int NIS = 2;                       // input stages
   static constexpr int VCOL = GP * NT;                // first V column in TMEM
   static constexpr int TMEM_COLS = 512;
   static constexpr int UBYTES = GP * 2 * NT * 32;     // one k-step of U (GP points, hi+lo)
-  static constexpr int NTHREADS = tc_threads(GP);
+  static constexpr int NTHREADS = tc_threads(GP, NT);
   static constexpr int PPI = GP / NISS;               // points per issuer
   static_assert(A % GP == 0 && GP % 2 == 0, "passes must hold whole ± pairs");
   static_assert(NS >= 2 && NS % NWG == 0, "stage ring");
@@ -97,22 +96,26 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT>::NTHREADS, 1)
   using Cfg = TcCfg<M, RW, NT>;
   using T = typename Cfg::T;
   constexpr int A = Cfg::A, GP = Cfg::GP, NS = Cfg::NS, NISS = Cfg::NISS, NWG = Cfg::NWG;
-  constexpr int NPASS = Cfg::NPASS, NIS = Cfg::NIS, VCOL = Cfg::VCOL, PPI = Cfg::PPI;
+  constexpr int NPASS = Cfg::NPASS, VCOL = Cfg::VCOL, PPI = Cfg::PPI;
+  const int NIS = pl.NIS;  // input stages (runtime: fills the shared-memory budget)
   constexpr uint32_t UBYTES = Cfg::UBYTES;
 
   extern __shared__ __align__(1024) uint8_t smem[];
   const uint32_t inplane = (uint32_t)pl.PLANE;  // plane stride (128-aligned)
-  uint8_t* u_smem = smem;                                        // [NS][UBYTES]
-  uint8_t* in_smem = u_smem + (size_t)NS * UBYTES;               // [NIS][2 planes][PLANE]
-  uint8_t* o_smem = in_smem + (size_t)NIS * 2 * inplane;         // [NWG][NOB][OSTRIDE]
-  uint64_t* bars = reinterpret_cast<uint64_t*>(o_smem + (size_t)NWG * pl.NOB * pl.OSTRIDE);
+  const int NUS = pl.NUS;  // U ring slots (runtime: deeper than the TMEM V stages to hide L2 latency)
+  uint8_t* u_smem = smem;                                        // [NUS][UBYTES]         (1024-aligned)
+  uint8_t* o_smem = u_smem + (size_t)NUS * UBYTES;               // [NWG][NOB][OSTRIDE]   (1024-aligned)
+  uint8_t* in_smem = o_smem + (size_t)NWG * pl.NOB * pl.OSTRIDE;  // [NIS][2 planes][PLANE]
+  uint64_t* bars = reinterpret_cast<uint64_t*>(in_smem + (size_t)NIS * 2 * inplane);
   uint64_t* in_full = bars;             // [NIS]
   uint64_t* in_empty = in_full + NIS;   // [NIS]
   uint64_t* st_full = in_empty + NIS;   // [NS]
   uint64_t* st_empty = st_full + NS;    // [NS]
   uint64_t* d_full = st_empty + NS;     // [1]
   uint64_t* d_empty = d_full + 1;       // [1]
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(d_empty + 1);
+  uint64_t* u_full = d_empty + 1;       // [NUS]
+  uint64_t* u_empty = u_full + NUS;     // [NUS]
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(u_empty + NUS);
 
   const int warp = threadIdx.x / 32, lane32 = threadIdx.x % 32;
   const int b = blockIdx.x;
@@ -123,11 +126,12 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT>::NTHREADS, 1)
   const int rb = tb % pl.PB;
   const int n = tb / pl.PB;
   const int p0 = rb * pl.ROWS;
-  constexpr int PROD_WARP = NWG * 4, ISS_WARP0 = NWG * 4 + 1;
+  constexpr int PROD_WARP = NWG * 4, UPROD_WARP = NWG * 4 + 1, ISS_WARP0 = NWG * 4 + 2;
 
   if (threadIdx.x == 0) {
     for (int i = 0; i < NIS; ++i) { mbar_init(&in_full[i], 1); mbar_init(&in_empty[i], NWG * 128); }
-    for (int i = 0; i < NS; ++i) { mbar_init(&st_full[i], 128 + 1); mbar_init(&st_empty[i], NISS); }
+    for (int i = 0; i < NS; ++i) { mbar_init(&st_full[i], 128); mbar_init(&st_empty[i], NISS); }
+    for (int i = 0; i < NUS; ++i) { mbar_init(&u_full[i], 1); mbar_init(&u_empty[i], NISS); }
     mbar_init(d_full, NISS);
     mbar_init(d_empty, NWG * 128);
     fence_mbar_init();
@@ -152,20 +156,28 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT>::NTHREADS, 1)
     const uint32_t lane_addr = tbase + ((uint32_t)(l & ~31) << 16);
     const int TSM = pl.TS * M;  // output columns per CTA row segment
     float* ostage = reinterpret_cast<float*>(o_smem + (size_t)g * pl.NOB * pl.OSTRIDE);
+    // staged row of this tile in the output box (box order: channels, tiles, rows) and its
+    // TMA swizzle: 128B rows (CPW = 32) XOR chunk with r & 7; 64B rows (CPW = 16) with (r>>1) & 3
+    constexpr int CPW = NT / NWG;
+    const int orow = has_slot ? row_l * pl.TS + tw_l : 0;
+    const int oswz = CPW == 32 ? (orow & 7) : ((orow >> 1) & 3);
 
+    int ist = 0, iph = 0;  // input ring slot / phase (incremental: no runtime division)
     static_for<NPASS>([&](auto PASS_) {
       constexpr int PASS = PASS_;
       for (int cc = 0; cc < pl.NCC; ++cc) {
-        const int li = PASS * pl.NCC + cc, ist = li % NIS;
-        mbar_wait(&in_full[ist], (li / NIS) & 1);
+        const int li = PASS * pl.NCC + cc;
+        if (l == 0) trace_rec(pl.trace, 19 + g, li);
+        mbar_wait(&in_full[ist], iph);
+        if (l == 0) trace_rec(pl.trace, 23 + g, li);
         const float4* planes = reinterpret_cast<const float4*>(in_smem + (size_t)ist * 2 * inplane);
         for (int fh = 0; fh < pl.R; ++fh) {
           const int kg = PASS * NKS + cc * pl.R + fh;  // global k-step index
           if (kg % NWG != g) continue;
           const int s = kg % NS, use = kg / NS;
-          if (l == 0) trace_rec(pl.trace, 3 * g + 0, kg / NWG);
+          if (l == 0) trace_rec(pl.trace, 0 + g, kg / NWG);
           if (use > 0) mbar_wait(&st_empty[s], (use - 1) & 1);
-          if (l == 0) trace_rec(pl.trace, 3 * g + 1, kg / NWG);
+          if (l == 0) trace_rec(pl.trace, 4 + g, kg / NWG);
           const uint32_t vbase = lane_addr + VCOL + s * GP * 16;
           const int off = (has_slot ? (row_l + fh) : 0) * pl.WBOX + col0;
 #pragma unroll
@@ -213,104 +225,117 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT>::NTHREADS, 1)
           tmem_wait_st();
           tc_fence_before();
           mbar_arrive(&st_full[s]);
-          if (l == 0) trace_rec(pl.trace, 3 * g + 2, kg / NWG);
+          if (l == 0) trace_rec(pl.trace, 8 + g, kg / NWG);
+          if (g == 0 && (l & 31) == 0) trace_rec(pl.trace, 12 + (l >> 5), kg / NWG);
         }
         mbar_arrive(&in_empty[ist]);
+        if (++ist == NIS) { ist = 0; iph ^= 1; }
       }
       // ---------- epilogue of this pass: y (+)= A^T M via shared memory + TMA ----------
-      if (l == 0) trace_rec(pl.trace, 8 + g, 2 * PASS);
+      if (l == 0 && g == 0) trace_rec(pl.trace, 27, 2 * PASS);
       mbar_wait(d_full, PASS & 1);
       tc_fence_after();
-      if (l == 0) trace_rec(pl.trace, 8 + g, 2 * PASS + 1);
-      constexpr int CPW = NT / NWG;
+      if (l == 0 && g == 0) trace_rec(pl.trace, 27, 2 * PASS + 1);
+      // One output column i at a time over this warpgroup's CPW channels: every tile's
+      // y[q0 + i][cbase .. cbase+CPW) is one 128-byte (64-byte) row of the staging box,
+      // and the TMA store walks Q with element stride m (positions q0 + i of all tiles).
       const int qbase = seg * TSM;
-#pragma unroll 1
-      for (int c8 = 0; c8 < CPW / 8; ++c8) {
-        const int col = g * CPW + c8 * 8;
-        float Mt[GP][8];
-#pragma unroll
-        for (int tl = 0; tl < GP; ++tl) tmem_ld_x8(lane_addr + tl * NT + col, Mt[tl]);
-        tmem_wait_ld();
-        if (c8 == CPW / 8 - 1) {  // accumulators fully read: the issuers may start the next pass
-          tc_fence_before();
-          mbar_arrive(d_empty);
-        }
+      const int cbase = g * CPW;
+      static_for<M>([&](auto I_) {
+        constexpr int i = I_;
         // staging buffer reuse: the TMA store that last read it must be done reading
-        const int ob = pl.NOB == 2 ? (c8 & 1) : 0;
+        const int ob = i % pl.NOB;
         if (l == 0) {
           if (pl.NOB == 2) bulk_wait_group_read<1>();
           else bulk_wait_group_read<0>();
         }
         named_bar_sync(1 + g, 128);
-        float* stg = ostage + (size_t)ob * (pl.OSTRIDE / 4);
-        static_for<M>([&](auto I_) {
-          constexpr int i = I_;
-          float o[8];
+        float4* stg = reinterpret_cast<float4*>(ostage + (size_t)ob * (pl.OSTRIDE / 4)) + (size_t)orow * (CPW / 4);
+#pragma unroll 1
+        for (int hh = 0; hh < CPW / 16; ++hh) {  // 16 channels at a time (register budget)
+          float o[16];
 #pragma unroll
-          for (int e = 0; e < 8; ++e) o[e] = 0.f;
+          for (int e = 0; e < 16; ++e) o[e] = 0.f;
           static_for<GP / 2>([&](auto Q_) {
-            constexpr int idx0 = PASS * GP + 2 * (int)Q_;
+            constexpr int idx0 = PASS * GP + 2 * (int)Q_;  // pair slot (internal points idx0, idx0+1)
             constexpr int tl0 = 2 * (int)Q_;
+            float ma[16], mb[16];
+            tmem_ld_x16(lane_addr + tl0 * NT + cbase + 16 * hh, ma);
+            tmem_ld_x16(lane_addr + (tl0 + 1) * NT + cbase + 16 * hh, mb);
+            tmem_wait_ld();
             if constexpr (idx0 == 0) {
               constexpr float c0 = T::AT(i, 0), c1 = T::AT(i, A - 1);
 #pragma unroll
-              for (int e = 0; e < 8; ++e) {
-                if constexpr (c0 != 0.f) o[e] = fmaf(c0, Mt[tl0][e], o[e]);
-                if constexpr (c1 != 0.f) o[e] = fmaf(c1, Mt[tl0 + 1][e], o[e]);
+              for (int e = 0; e < 16; ++e) {
+                if constexpr (c0 != 0.f) o[e] = fmaf(c0, ma[e], o[e]);
+                if constexpr (c1 != 0.f) o[e] = fmaf(c1, mb[e], o[e]);
               }
-            } else {
+            } else {  // AT[i][a+1] = (-1)^i AT[i][a] (pair structure)
               constexpr int pa = point_of(idx0, A);
               constexpr float ca = T::AT(i, pa);
 #pragma unroll
-              for (int e = 0; e < 8; ++e) {
-                const float sv = (i % 2 == 0) ? (Mt[tl0][e] + Mt[tl0 + 1][e]) : (Mt[tl0][e] - Mt[tl0 + 1][e]);
+              for (int e = 0; e < 16; ++e) {
+                const float sv = (i % 2 == 0) ? (ma[e] + mb[e]) : (ma[e] - mb[e]);
                 if constexpr (ca == 1.f) o[e] += sv;
                 else if constexpr (ca != 0.f) o[e] = fmaf(ca, sv, o[e]);
               }
             }
           });
           if (has_slot) {
-            float4* dst = reinterpret_cast<float4*>(stg + ((size_t)row_l * TSM + tw_l * M + i) * 8);
-            dst[0] = make_float4(o[0], o[1], o[2], o[3]);
-            dst[1] = make_float4(o[4], o[5], o[6], o[7]);
+#pragma unroll
+            for (int j = 0; j < 4; ++j)
+              stg[(4 * hh + j) ^ oswz] = make_float4(o[4 * j], o[4 * j + 1], o[4 * j + 2], o[4 * j + 3]);
           }
-        });
+        }
+        if constexpr (i == M - 1) {  // accumulators fully read: the issuers may start the next pass
+          tc_fence_before();
+          mbar_arrive(d_empty);
+        }
         fence_proxy_async_smem();
         named_bar_sync(1 + g, 128);
         if (l == 0) {
-          const int k0 = nb * NT + col;
-          if constexpr (PASS == 0) tma_store_4d(&ymap, stg, k0, qbase, p0, n);
-          else tma_reduce_add_4d(&ymap, stg, k0, qbase, p0, n);
+          const float* box = ostage + (size_t)ob * (pl.OSTRIDE / 4);
+          const int k0 = nb * NT + cbase;
+          if constexpr (PASS == 0) tma_store_4d(&ymap, box, k0, qbase + i, p0, n);
+          else tma_reduce_add_4d(&ymap, box, k0, qbase + i, p0, n);
           bulk_commit_group();
         }
-      }
+      });
       // this pass's writes must be complete before the next pass's reduce-add
       if (l == 0) bulk_wait_group_all();
-      if (l == 0) trace_rec(pl.trace, 10 + g, PASS);
+      if (l == 0 && g == 0) trace_rec(pl.trace, 28, PASS);
     });
   } else if (warp == PROD_WARP) {
-    // ====================== TMA / bulk-copy producer ======================
+    // ====================== input-row TMA producer ======================
     if (lane32 == 0) {
       tma_prefetch_desc(&xmap);
       tma_prefetch_desc(&ymap);
       const int wstart = seg * pl.TS * M - pl.pad_w;
       const int hstart = p0 - pl.pad_h;
+      int ist = 0, iph = 0, first = 1;  // slot, round parity, still in the first round
       for (int pass = 0; pass < NPASS; ++pass) {
         for (int cc = 0; cc < pl.NCC; ++cc) {
-          const int li = pass * pl.NCC + cc, ist = li % NIS;
-          if (li >= NIS) mbar_wait(&in_empty[ist], ((li / NIS) - 1) & 1);
+          if (!first) mbar_wait(&in_empty[ist], iph ^ 1);
           uint8_t* dst = in_smem + (size_t)ist * 2 * inplane;
           mbar_expect_tx(&in_full[ist], 2u * (uint32_t)pl.BOXB);
           tma_load_4d(dst, &xmap, &in_full[ist], cc * 8, wstart, hstart, n);
           tma_load_4d(dst + inplane, &xmap, &in_full[ist], cc * 8 + 4, wstart, hstart, n);
-          for (int fh = 0; fh < pl.R; ++fh) {
-            const int ks = cc * pl.R + fh, kg = pass * NKS + ks;
-            const int s = kg % NS, use = kg / NS;
-            if (use > 0) mbar_wait(&st_empty[s], (use - 1) & 1);
-            mbar_expect_tx(&st_full[s], UBYTES);
-            bulk_load(u_smem + (size_t)s * UBYTES, u + u_offset(NT, A, nb, NKS, ks, pass * GP, 0), UBYTES,
-                      &st_full[s]);
-          }
+          if (++ist == NIS) { ist = 0; iph ^= 1; first = 0; }
+        }
+      }
+    }
+    __syncwarp();
+  } else if (warp == UPROD_WARP) {
+    // ======================= U (transformed filter) ring =======================
+    if (lane32 == 0) {
+      int us = 0, uph = 0, first = 1;
+      for (int pass = 0; pass < NPASS; ++pass) {
+        const float* src = u + u_offset(NT, A, nb, NKS, 0, pass * GP, 0);
+        for (int ks = 0; ks < NKS; ++ks, src += (size_t)A * 2 * NT * 8) {
+          if (!first) mbar_wait(&u_empty[us], uph ^ 1);
+          mbar_expect_tx(&u_full[us], UBYTES);
+          bulk_load(u_smem + (size_t)us * UBYTES, src, UBYTES, &u_full[us]);
+          if (++us == NUS) { us = 0; uph ^= 1; first = 0; }
         }
       }
     }
@@ -320,20 +345,22 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT>::NTHREADS, 1)
     const int iss = warp - ISS_WARP0;  // owns points tl = iss * PPI .. iss * PPI + PPI - 1
     if (lane32 == 0) {
       constexpr uint32_t idesc = idesc_tf32(128, NT);
-      const uint32_t u_base = smem_u32(u_smem);
+      // descriptor of U slot 0, point 0, hi; other images = + (byte offset >> 4) in the start field
+      const uint64_t bdesc0 = umma_desc_kmajor_noswizzle(smem_u32(u_smem), NT * 16, 128);
+      int s = 0, sph = 0, us = 0, uph = 0;  // V stage / U slot and their round parities
+      int kg = 0;
       for (int pass = 0; pass < NPASS; ++pass) {
         if (pass > 0) {
           mbar_wait(d_empty, (pass - 1) & 1);
           tc_fence_after();
         }
-        for (int ks = 0; ks < NKS; ++ks) {
-          const int kg = pass * NKS + ks;
-          const int s = kg % NS, use = kg / NS;
-          if (iss == 0) trace_rec(pl.trace, 12, kg);
-          mbar_wait(&st_full[s], use & 1);
+        for (int ks = 0; ks < NKS; ++ks, ++kg) {
+          if (iss == 0) trace_rec(pl.trace, 29, kg);
+          mbar_wait(&st_full[s], sph);
+          mbar_wait(&u_full[us], uph);
           tc_fence_after();
-          if (iss == 0) trace_rec(pl.trace, 6, kg);
-          const uint32_t ub = u_base + s * UBYTES;
+          if (iss == 0) trace_rec(pl.trace, 16, kg);
+          const uint64_t bslot = bdesc0 + (uint64_t)((us * UBYTES) >> 4);
           const uint32_t va = tbase + VCOL + s * GP * 16;
           // product order lo*hi, hi*lo, hi*hi (small terms first), points innermost
 #pragma unroll
@@ -342,13 +369,16 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT>::NTHREADS, 1)
             for (int pi = 0; pi < PPI; ++pi) {
               const int tl = iss * PPI + pi;
               const uint32_t a = va + tl * 16 + (prod == 0 ? 8 : 0);
-              const uint64_t bd = umma_desc_kmajor_noswizzle(ub + (tl * 2 + (prod == 1 ? 1 : 0)) * NT * 32, NT * 16, 128);
+              const uint64_t bd = bslot + (uint64_t)(((tl * 2 + (prod == 1 ? 1 : 0)) * NT * 32) >> 4);
               mma_tf32_ts(tbase + tl * NT, a, bd, idesc, (ks > 0 || prod > 0) ? 1u : 0u);
             }
           }
-          if (iss == 0) trace_rec(pl.trace, 7, kg);
+          if (iss == 0) trace_rec(pl.trace, 17, kg);
           mma_commit(&st_empty[s]);
-          if (iss == 0) trace_rec(pl.trace, 14, kg);
+          mma_commit(&u_empty[us]);
+          if (iss == 0) trace_rec(pl.trace, 18, kg);
+          if (++s == NS) { s = 0; sph ^= 1; }
+          if (++us == NUS) { us = 0; uph ^= 1; }
         }
         mma_commit(d_full);
       }

@@ -1,11 +1,16 @@
-"""Diagnostic: CTA-0 timeline of the fused kernel (clock64 cycles) for one config."""
+"""Diagnostic: CTA-0 timeline of the fused kernel (clock64 cycles) for one config.
+Trace kinds (see trace_rec calls in fused_tc.cu): 0-3 WG k-step start, 4-7 after st_empty wait,
+8-11 after st_full arrive (warp 0 of each WG), 12-15 WG0 per-warp arrive, 16-18 issuer 0
+(after st_full wait, after issue, after commit), 19-22/23-26 WG in_full before/after,
+27 epilogue d_full wait (before/after), 28 epilogue end, 29 issuer 0 before st_full wait."""
 import ctypes, os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np, torch
 import paper_conf_icpp_zhangzxyw24_b200 as i2cw
 
 cfgs = {"cfg2": ("conv", 128, 56, 56, 64, 64, 3, 3, 1, 1), "r9": ("conv", 64, 32, 32, 128, 128, 9, 9, 4, 4),
-        "r5": ("conv", 64, 32, 32, 128, 128, 5, 5, 2, 2), "c512": ("conv", 256, 28, 28, 512, 512, 3, 3, 1, 1)}
+        "r5": ("conv", 64, 32, 32, 128, 128, 5, 5, 2, 2), "r3": ("conv", 64, 32, 32, 128, 128, 3, 3, 1, 1),
+        "c512": ("conv", 256, 28, 28, 512, 512, 3, 3, 1, 1)}
 L = i2cw.lib()
 L.i2cw_debug_trace.argtypes = [ctypes.c_int] * 10 + [ctypes.c_void_p] * 5
 for name in sys.argv[1:] or ["cfg2"]:
@@ -13,33 +18,41 @@ for name in sys.argv[1:] or ["cfg2"]:
     x = torch.rand((N, H, W, C), device="cuda"); w = torch.rand((K, R, S, C), device="cuda")
     P, Q = H + 2 * ph - R + 1, W + 2 * pw - S + 1
     y = torch.empty((N, P, Q, K), device="cuda")
-    tr = torch.zeros(16 * 512, dtype=torch.int64, device="cuda")
+    tr = torch.zeros(32 * 512, dtype=torch.int64, device="cuda")
     for _ in range(3):
         tr.zero_()
         rc = L.i2cw_debug_trace(0, N, H, W, C, K, R, S, ph, pw, x.data_ptr(), w.data_ptr(), y.data_ptr(), tr.data_ptr(),
                                 torch.cuda.current_stream().cuda_stream)
         assert rc == 0
     torch.cuda.synchronize()
-    t = tr.cpu().numpy().reshape(16, 512).astype(np.int64)
+    t = tr.cpu().numpy().reshape(32, 512).astype(np.int64)
     t0 = t[t > 0].min()
     t = np.where(t > 0, t - t0, -1)
-    def valid(k): return t[k][t[k] >= 0]
-    print(f"== {name}: plan {i2cw.debug_plan(kind, N, H, W, C, K, R, S, ph, pw)}")
-    for g in range(2):
-        a, b, c = valid(3 * g), valid(3 * g + 1), valid(3 * g + 2)
+    def v(k): return t[k][t[k] >= 0]
+    pl = i2cw.debug_plan(kind, N, H, W, C, K, R, S, ph, pw)
+    print(f"== {name}: plan {pl}")
+    nwg = 4 if pl["NT"] == 64 else 2
+    for g in range(nwg):
+        a, b, c = v(g), v(4 + g), v(8 + g)
         n = min(len(a), len(b), len(c))
-        print(f"WG{g}: {n} ksteps; wait(v_empty) med {np.median(b[:n]-a[:n]):.0f} cyc; transform med {np.median(c[:n]-b[:n]):.0f} cyc; "
-              f"period med {np.median(np.diff(a[:n])):.0f}")
-    r6, r7 = valid(6), valid(7)
-    n = min(len(r6), len(r7))
-    print(f"MMA: {n} ksteps; issue dur med {np.median(r7[:n]-r6[:n]):.0f}; ready->ready med {np.median(np.diff(r6[:n])):.0f} cyc; total span {r7[n-1]-r6[0]}")
-    for g in range(2):
-        e = valid(8 + g); f = valid(10 + g)
-        print(f"WG{g} epilogue: wait d_full at {e.tolist()}, done {f.tolist()}")
-    print("first 12 MMA ready times:", r6[:12].tolist())
-    print("first 6 WG0 (start, after-wait, arrive):", list(zip(valid(0)[:6].tolist(), valid(1)[:6].tolist(), valid(2)[:6].tolist())))
-    r12, r13, r14 = valid(12), valid(13), valid(14)
-    print("MMA thread per k-step: (start, after v_full, after u_full, issued, after commits) first 8:")
-    for i in range(8):
-        print("   ", r12[i], r13[i], r6[i], r7[i], r14[i])
-    print("WG1 first 6 (start, after-wait, arrive):", list(zip(valid(3)[:6].tolist(), valid(4)[:6].tolist(), valid(5)[:6].tolist())))
+        if n < 2: continue
+        print(f"WG{g}: {n} ks; st_empty wait med {np.median(b[:n]-a[:n]):.0f}; transform med {np.median(c[:n]-b[:n]):.0f}; "
+              f"arrive->next start med {np.median(a[1:n]-c[:n-1]):.0f}; period med {np.median(np.diff(a[:n])):.0f}")
+        fa, fb = v(19 + g), v(23 + g)
+        m = min(len(fa), len(fb))
+        print(f"      in_full waits med {np.median(fb[:m]-fa[:m]):.0f} max {np.max(fb[:m]-fa[:m])} sum {np.sum(fb[:m]-fa[:m])}")
+    w29, w16, w17, w18 = v(29), v(16), v(17), v(18)
+    n = min(len(w29), len(w16), len(w17), len(w18))
+    print(f"issuer0: {n} ks; st_full wait med {np.median(w16[:n]-w29[:n]):.0f}; issue med {np.median(w17[:n]-w16[:n]):.0f}; "
+          f"commit med {np.median(w18[:n]-w17[:n]):.0f}; ready->ready med {np.median(np.diff(w16[:n])):.0f}; span {w18[n-1]-w16[0]}")
+    arr = [v(12 + w) for w in range(4)]
+    n = min(len(a) for a in arr)
+    A_ = np.stack([a[:n] for a in arr])
+    print("WG0 per-warp arrive minus warp0 (median):", [float(np.median(A_[w] - A_[0])) for w in range(4)])
+    print("epilogue d_full wait (before, after):", v(27).tolist(), " end:", v(28).tolist())
+    # per k-step critical path sample: ks 8..15
+    print("kg: WG arrive(last warp of WG0 only for g=0) | issuer ready | issued | committed")
+    for kg in range(8, 16):
+        g = kg % nwg; i = kg // nwg
+        arrive = v(8 + g)[i] if i < len(v(8 + g)) else None
+        print(f"  {kg:3d} g{g} arrive {arrive}  ready {w16[kg]}  issued {w17[kg]}  commit {w18[kg]}")
