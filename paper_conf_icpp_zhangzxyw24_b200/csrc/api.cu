@@ -16,7 +16,7 @@
 
 namespace i2cw {
 cudaError_t launch_filter_transform(const float* w, float* u, int C, int K, int R, int S, int is_deconv, int alpha,
-                                    int NT, int NB, int NCC, const double* G, cudaStream_t stream);
+                                    int NT, int NB, int NCC, int halves, const double* G, cudaStream_t stream);
 cudaError_t launch_fused_tc(const CUtensorMap& xmap, const CUtensorMap& ymap, const Plan& pl, const float* u,
                             cudaStream_t stream);
 cudaError_t launch_fused_simt(const Plan& pl, const float* x, const float* u, float* y, cudaStream_t stream);
@@ -66,7 +66,10 @@ int assign_lanes(int ROWS, int TS, int WBOX, int m, int cpw, unsigned char* lrow
   for (int r = 0; r < ROWS; ++r)
     for (int t = 0; t < TS; ++t) {
       const int orow = r * TS + t;
-      pool.push_back({r, t, (r * WBOX + t * m) % 8, cpw == 32 ? (orow & 7) : ((orow >> 1) & 3)});
+      // 128B rows: bank group = chunk ^ (r & 7); 64B rows: (r & 1) * 4 + (chunk ^ ((r >> 1) & 3)).
+      // Either way 8 lanes with distinct r mod 8 hit 8 distinct bank groups.
+      (void)cpw;
+      pool.push_back({r, t, (r * WBOX + t * m) % 8, orow & 7});
     }
   std::fill(lrow, lrow + kMaxLanes, 0xFF);
   std::fill(ltw, ltw + kMaxLanes, 0);
@@ -91,7 +94,7 @@ int assign_lanes(int ROWS, int TS, int WBOX, int m, int cpw, unsigned char* lrow
     }
     int mi = 0, mo = 0;
     for (int i = 0; i < 8; ++i) { mi = std::max(mi, cin[i]); mo = std::max(mo, cout_[i]); }
-    cost += (mi - 1) + (cpw == 32 ? (mo - 1) : std::max(0, mo - 2));
+    cost += (mi - 1) + (mo - 1);
   }
   return cost;
 }
@@ -135,7 +138,14 @@ int make_plan(int N, int H, int W, int C, int K, int R, int S, int pad_h, int pa
   rows = std::min(rows, pl.P);
   rows = std::min(rows, 256 - (R - 1));
   if (rows < 1) return I2CW_EUNSUPPORTED;
-  const int ubytes = pl.GP * 2 * pl.NT * 32;
+  // CTA pairs (tcgen05.mma.cta_group::2, each CTA stages half of U): correct (all parity tests)
+  // but measured 2-4% slower than single CTAs at every config, so opt-in via I2CW_PAIR=1.
+  static const bool pair_ok = [] { const char* e = getenv("I2CW_PAIR"); return e && e[0] == '1'; }();
+  pl.pair = pair_ok ? 1 : 0;
+  // DEBUG timing ablation (never set in production; results are wrong when non-zero)
+  static const int ablate = [] { const char* e = getenv("I2CW_ABLATE"); return e ? atoi(e) : 0; }();
+  pl.ablate = ablate;
+  const int ubytes = pl.GP * 2 * pl.NT * 32 / (pl.pair ? 2 : 1);
   const int NS = ns_for(pl.alpha, pl.NT);
   pl.NUS = NS;
   pl.NOB = 2;
@@ -168,13 +178,14 @@ int make_plan(int N, int H, int W, int C, int K, int R, int S, int pad_h, int pa
     static const int kDepths[][3] = {{8, 3, 2}, {8, 3, 1}, {6, 3, 2}, {6, 3, 1}, {6, 2, 1},
                                      {4, 3, 1}, {4, 2, 1}, {3, 2, 1}, {2, 2, 1}};
     bool fit = false;
+    const int kps = kps_for(pl.alpha, pl.NT);  // k-steps per U super-slot
     for (const auto& d : kDepths) {
-      pl.NUS = std::max(d[0], NS);
+      pl.NUS = std::max(d[0] / kps, 2);  // U super-slots
       pl.NIS = d[1];
       pl.NOB = d[2];
-      const int bar_bytes = 8 * (2 * pl.NIS + 2 * NS + 2 + 2 * pl.NUS) + 16;
-      pl.smem_bytes =
-          pl.NUS * ubytes + pl.NIS * 2 * pl.PLANE + nwg_for(pl.NT) * pl.NOB * pl.OSTRIDE + bar_bytes;
+      const int bar_bytes = 8 * (2 * pl.NIS + 3 * (NS / kps) + 2 + 2 * pl.NUS) + 16;
+      pl.smem_bytes = pl.NUS * kps * ubytes + pl.NIS * 2 * pl.PLANE + nwg_for(pl.NT) * pl.NOB * pl.OSTRIDE +
+                      bar_bytes;
       if (pl.smem_bytes <= kSmemBudget) { fit = true; break; }
     }
     if (fit) break;
@@ -302,11 +313,12 @@ int transform_into(const Plan& pl, int is_deconv, const float* w, void* u, cudaS
   std::memset(&tag, 0, sizeof(tag));
   tag.magic = kUMagic; tag.alpha = pl.alpha; tag.m = pl.m; tag.is_deconv = is_deconv;
   tag.C = pl.C; tag.K = pl.K; tag.R = pl.R; tag.S = pl.S; tag.NT = pl.NT; tag.NB = pl.NB; tag.NCC = pl.NCC;
+  tag.halves = pl.pair ? 2 : 1;
   static_assert(sizeof(UTag) <= kUTagBytes, "tag");
   if (cudaMemcpyAsync(u, &tag, sizeof(tag), cudaMemcpyHostToDevice, stream) != cudaSuccess) return I2CW_ECUDA;
   registry_put(u, tag);
   float* ud = reinterpret_cast<float*>(static_cast<uint8_t*>(u) + kUTagBytes);
-  if (launch_filter_transform(w, ud, pl.C, pl.K, pl.R, pl.S, is_deconv, pl.alpha, pl.NT, pl.NB, pl.NCC, G.data(),
+  if (launch_filter_transform(w, ud, pl.C, pl.K, pl.R, pl.S, is_deconv, pl.alpha, pl.NT, pl.NB, pl.NCC, pl.pair ? 2 : 1, G.data(),
                               stream) != cudaSuccess)
     return I2CW_ECUDA;
   return I2CW_OK;
@@ -329,6 +341,7 @@ int conv_common(int is_deconv, int N, int H, int W, int C, int K, int R, int S, 
   int rc = make_plan(N, H, W, C, K, R, S, pad_h, pad_w, is_deconv, &pl);
   if (rc != I2CW_OK) return rc;
   pl.trace = trace;
+  if (simt) pl.pair = 0;  // the SIMT stepping stone reads the single-CTA U layout
   if ((rc = bind_device_of(x)) != I2CW_OK) return rc;
   void* u = nullptr;
   const size_t ub = kUTagBytes + u_data_bytes(pl);
@@ -365,7 +378,8 @@ int pretransformed_common(int is_deconv, int N, int H, int W, int C, int K, int 
     }
   }
   if (tag.magic != kUMagic || (int)tag.is_deconv != is_deconv || (int)tag.C != C || (int)tag.K != K ||
-      (int)tag.R != R || (int)tag.S != S || (int)tag.alpha != pl.alpha || (int)tag.m != pl.m || (int)tag.NT != pl.NT)
+      (int)tag.R != R || (int)tag.S != S || (int)tag.alpha != pl.alpha || (int)tag.m != pl.m || (int)tag.NT != pl.NT ||
+      (int)tag.halves != (pl.pair ? 2 : 1))
     return I2CW_EINVAL;
   rc = run_fused(pl, x, u, y, stream);
   if (rc != I2CW_OK) cudaGetLastError();

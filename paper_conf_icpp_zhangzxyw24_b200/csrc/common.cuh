@@ -37,6 +37,9 @@ struct Plan {
   int NOB;              // output staging buffers per warpgroup (1 or 2)
   int NIS;              // input (x row box) stages
   int smem_bytes;
+  int pair;             // 1: CTA pairs (cluster of 2) with tcgen05.mma.cta_group::2, U split by N halves
+  int ablate;           // DEBUG timing ablation (I2CW_ABLATE, results wrong): 1 no transform math,
+                        // 2 no MMAs, 4 no epilogue math/stores; 0 in production
   unsigned long long* trace;  // debug timeline of CTA 0 (nullptr = off), see i2cw_debug_trace
   unsigned char lane_row[kMaxLanes];  // lane -> row within block (0xFF = idle lane)
   unsigned char lane_tw[kMaxLanes];   // lane -> tile within segment
@@ -54,6 +57,8 @@ __host__ __device__ constexpr int ns_for(int alpha, int NT) {
              ? 4
              : (((512 - gp_for(alpha, NT) * NT) / (gp_for(alpha, NT) * 16)) / 2) * 2;
 }
+// k-steps per super-stage (one barrier round trip + one U slot): 2 when 4 V slots fit
+__host__ __device__ constexpr int kps_for(int alpha, int NT) { return ns_for(alpha, NT) >= 4 ? 2 : 1; }
 // MMA-issuing warps: one warp issues at most ~1 UMMA per 45 cycles (measured,
 // tools/mma_bench.cu), so several warps issue, each owning whole accumulators.
 __host__ __device__ constexpr int niss_for(int GP) { return GP % 4 == 0 ? 4 : (GP % 3 == 0 ? 3 : 2); }
@@ -79,16 +84,29 @@ __host__ __device__ inline size_t u_offset(int NT, int alpha, int nb, int NKS, i
   return ((((size_t)nb * NKS + ks) * alpha + idx) * 2 + hl) * (size_t)NT * 8;
 }
 
+// CTA-pair layout (Plan::pair): the N rows of every image are split in two halves owned
+// by the two CTAs of a cluster; per (nb, ks) the halves are outermost so one CTA's share of
+// a pass is one contiguous run:  U[nb][ks][h][idx][hl][kc][n'][e],  n' < NT/2.
+// Returns the offset of image (nb, ks, h, idx, hl = 0); hl = 1 follows at + (NT/2)*8.
+__host__ __device__ inline size_t u_offset_pair(int NT, int alpha, int nb, int NKS, int ks, int h, int idx) {
+  return (((((size_t)nb * NKS + ks) * 2 + h) * alpha + idx) * 2) * (size_t)(NT / 2) * 8;
+}
+
 constexpr int kUTagBytes = 256;
 constexpr uint32_t kUMagic = 0x49324357u;  // "I2CW"
 struct UTag {
-  uint32_t magic, alpha, m, is_deconv, C, K, R, S, NT, NB, NCC, pad;
+  uint32_t magic, alpha, m, is_deconv, C, K, R, S, NT, NB, NCC, halves;
 };
 
 #if defined(__CUDACC__)
-// Debug timeline: kind k, entry i -> trace[k * 512 + i] = clock64 (CTA 0 only).
+// Debug timeline: CTA b < 2, kind k, entry i -> trace[(b * 32 + k) * 512 + i] = globaltimer (ns;
+// comparable across the two SMs of a CTA pair).
 __device__ __forceinline__ void trace_rec(unsigned long long* tr, int kind, int i) {
-  if (tr != nullptr && blockIdx.x == 0 && i < 512) tr[kind * 512 + i] = clock64();
+  if (tr != nullptr && blockIdx.x < 2 && i < 512) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    tr[(blockIdx.x * 32 + kind) * 512 + i] = t;
+  }
 }
 // ----------------------------------------------------------------------------
 // PTX helpers
@@ -188,7 +206,83 @@ __device__ __forceinline__ void bulk_load(void* smem_dst, const void* gsrc, uint
       : "memory");
 }
 
+// ---- clusters (CTA pairs for cta_group::2) ---------------------------------
+__device__ __forceinline__ uint32_t cluster_ctarank() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+  return r;
+}
+__device__ __forceinline__ void cluster_sync_all() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+// shared::cluster address of the same shared variable in CTA `rank` of the cluster
+__device__ __forceinline__ uint32_t mapa_shared(const void* p, uint32_t rank) {
+  uint32_t r;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(smem_u32(p)), "r"(rank));
+  return r;
+}
+// Remote arrive on the peer CTA's barrier. Relaxed: every use forwards the completion of
+// work that is already complete and visible to the tensor core (tcgen05.wait::st by the
+// writers, TMA complete_tx), observed through a local barrier wait; a release.cluster
+// arrive measured ~600 ns per call and paced the whole CTA pair.
+__device__ __forceinline__ void mbar_arrive_remote(uint32_t cluster_addr) {
+  asm volatile("mbarrier.arrive.relaxed.cluster.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
+}
+// parity wait with cluster-scope acquire, for barriers completed by the other CTA of a pair
+// (remote mbarrier arrives, multicast tcgen05.commit). Measured: a suspended try_wait is
+// not woken promptly by remote arrivals (waits of 2.5-4 us instead of ~0.1), so the
+// suspend time is capped with an explicit 64 ns hint.
+__device__ __forceinline__ bool mbar_try_wait_cluster(uint64_t* bar, uint32_t parity) {
+  uint32_t ok;
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 p, [%1], %2, %3;\n\t"
+      "selp.u32 %0, 1, 0, p;\n\t}"
+      : "=r"(ok)
+      : "r"(smem_u32(bar)), "r"(parity), "r"(64u)
+      : "memory");
+  return ok != 0;
+}
+__device__ __forceinline__ void mbar_wait_cluster(uint64_t* bar, uint32_t parity) {
+  if (mbar_try_wait_cluster(bar, parity)) return;
+  const uint64_t t0 = globaltimer();
+  while (!mbar_try_wait_cluster(bar, parity)) {
+    if (globaltimer() - t0 > 4000000000ull) __trap();
+  }
+}
+
 // ---- tcgen05 --------------------------------------------------------------
+__device__ __forceinline__ void tmem_alloc2(uint32_t* smem_dst, uint32_t ncols) {
+  asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(smem_dst)),
+               "r"(ncols)
+               : "memory");
+}
+__device__ __forceinline__ void tmem_relinquish2() {
+  asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;" ::: "memory");
+}
+__device__ __forceinline__ void tmem_dealloc2(uint32_t taddr, uint32_t ncols) {
+  asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(taddr), "r"(ncols) : "memory");
+}
+// D[tmem] (+)= A[tmem] * B[smem]^T over a CTA pair: M = 256 (128 rows per CTA, A and D
+// at the same TMEM address in both), B split along N (N/2 rows per CTA, same smem offset)
+__device__ __forceinline__ void mma2_tf32_ts(uint32_t d_tmem, uint32_t a_tmem, uint64_t b_desc, uint32_t idesc,
+                                             uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::2.kind::tf32 [%0], [%1], %2, %3, p;\n\t}" ::"r"(d_tmem),
+      "r"(a_tmem), "l"(b_desc), "r"(idesc), "r"(accumulate)
+      : "memory");
+}
+// commit of this thread's prior cta_group::2 MMAs to the barrier at the same smem
+// offset in both CTAs of the pair
+__device__ __forceinline__ void mma_commit2(uint64_t* bar) {
+  asm volatile(
+      "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(
+          smem_u32(bar)),
+      "h"((uint16_t)0x3)
+      : "memory");
+}
 __device__ __forceinline__ void tmem_alloc(uint32_t* smem_dst, uint32_t ncols) {
   asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(smem_dst)),
                "r"(ncols)

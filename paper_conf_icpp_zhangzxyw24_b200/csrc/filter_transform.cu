@@ -21,7 +21,8 @@ struct GTable {
 };
 
 __global__ void filter_transform_kernel(const float* __restrict__ w, float* __restrict__ u, int C, int K, int R,
-                                        int S, int is_deconv, int alpha, int NT, int NB, int NCC, GTable gt) {
+                                        int S, int is_deconv, int alpha, int NT, int NB, int NCC, int halves,
+                                        GTable gt) {
   const int NKS = NCC * R;
   const size_t total = (size_t)NB * NKS * alpha * 2 * NT * 4;  // (nb, ks, idx, kc, n, e)
   for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < total; i += (size_t)gridDim.x * blockDim.x) {
@@ -46,14 +47,21 @@ __global__ void filter_transform_kernel(const float* __restrict__ w, float* __re
       hi = tf32_rna(uv);
       lo = tf32_rna(uv - hi);
     }
-    const size_t base = u_offset(NT, alpha, nb, NKS, ks, idx, 0) + (size_t)kc * NT * 4 + (size_t)n * 4 + e;
-    u[base] = hi;
-    u[base + (size_t)NT * 8] = lo;  // hl = 1 image follows the hl = 0 image
+    if (halves == 2) {  // CTA-pair layout: [h][idx][hl][kc][n'][e] per (nb, ks)
+      const int hN = NT / 2, h = n / hN, n2 = n % hN;
+      const size_t base = u_offset_pair(NT, alpha, nb, NKS, ks, h, idx) + (size_t)kc * hN * 4 + (size_t)n2 * 4 + e;
+      u[base] = hi;
+      u[base + (size_t)hN * 8] = lo;
+    } else {
+      const size_t base = u_offset(NT, alpha, nb, NKS, ks, idx, 0) + (size_t)kc * NT * 4 + (size_t)n * 4 + e;
+      u[base] = hi;
+      u[base + (size_t)NT * 8] = lo;  // hl = 1 image follows the hl = 0 image
+    }
   }
 }
 
 cudaError_t launch_filter_transform(const float* w, float* u, int C, int K, int R, int S, int is_deconv, int alpha,
-                                    int NT, int NB, int NCC, const double* G /* alpha x S, internal order */,
+                                    int NT, int NB, int NCC, int halves, const double* G /* alpha x S, internal order */,
                                     cudaStream_t stream) {
   GTable gt;
   for (int i = 0; i < 16 * 9; ++i) gt.g[i] = 0.0;
@@ -63,7 +71,7 @@ cudaError_t launch_filter_transform(const float* w, float* u, int C, int K, int 
   int blocks = (int)((total + 255) / 256);
   if (blocks > 148 * 16) blocks = 148 * 16;
   if (blocks < 1) blocks = 1;
-  filter_transform_kernel<<<blocks, 256, 0, stream>>>(w, u, C, K, R, S, is_deconv, alpha, NT, NB, NCC, gt);
+  filter_transform_kernel<<<blocks, 256, 0, stream>>>(w, u, C, K, R, S, is_deconv, alpha, NT, NB, NCC, halves, gt);
   return cudaGetLastError();
 }
 

@@ -1,0 +1,540 @@
+// The fused Im2col-Winograd forward kernel for sm_100a (rows a2-a5 of
+// SURVEY.md §8(a)); deconvolution runs through the same kernel with a
+// rotated, channel-transposed U (filter_transform.cu).
+//
+// Method (§4.1, Fig 2): Stage 1 im2col is an index map;
+// Stage 2 slides 1D windows of alpha = m + S - 1 input columns along W, runs
+// F(m, S) on them and accumulates over filter rows fh and channels c:
+//   V_t[tile][(fh,c)] = sum_j BT[t][j] x[n][p-ph+fh][q0-pw+j][c]          (a3)
+//   M_t[tile][k]      = sum_{fh,c} V_t[tile][(fh,c)] U_t[k][(fh,c)]        (a4)
+//   y[n][p][q0+i][k]  = sum_t AT[i][t] M_t[tile][k]   (q0+i < Q only)      (a5)
+// A^T is applied once after the (fh, c) sum by linearity.
+//
+// B200 mapping:
+//  * CTA = 128 Winograd tiles (UMMA M, one TMEM lane each) x NT output channels.
+//    Tiles are ROWS output rows x TS tiles of one image; lane->tile is a host
+//    permutation that spreads the 16-byte shared-memory reads over banks.
+//  * a2: a TMA warp stages, per 8-channel chunk, the (ROWS+R-1) x WBOX input
+//    rows of the block as two 16-byte channel planes (OOB zero fill = padding,
+//    PAPER.md:337-338); the rows are reused across all fh (vertical overlap)
+//    and by neighbouring windows (the (r-1) horizontal overlap, §5.4).
+//    The same warp streams each k-step's U image (1D bulk copy) into a ring.
+//  * a3: NWG transform warpgroups (thread = tile) read the alpha-window from
+//    shared memory, apply BT with zeros/±1 folded at compile time and the ±
+//    pair trick, split 3xTF32 hi/lo and write V into TMEM
+//    with tcgen05.st (V is the UMMA A operand, "TS" mode: no SMEM read for A).
+//  * a4: NISS issuer warps, each owning GP/NISS points' accumulators, issue per
+//    k-step 3 tcgen05.mma.kind::tf32 per point (lo*hi, hi*lo, hi*hi). Several
+//    issuers are needed: one warp issues at most one UMMA per ~45 cycles while
+//    a 128x64x8 tf32 UMMA takes 32 (tools/mma_bench.cu). Each accumulator has
+//    exactly one issuer, so results are bitwise deterministic.
+//  * k-step stages: NS slots, each = V (TMEM) + U (SMEM); one "full" barrier
+//    (128 transform arrivals + U tx bytes) and one "empty" barrier (NISS commits).
+//  * a5: the warpgroups tcgen05.ld the accumulators, apply A^T in registers
+//    (pair trick), stage 8-channel slices in shared memory and TMA-store them
+//    (TMA clips q >= Q, p >= P, k >= K: the in-kernel boundary). Passes > 0 use a
+//    TMA reduce-add into y (the accumulators hold GP of alpha points per pass).
+#pragma once
+#include <utility>
+
+#include "common.cuh"
+#include "transforms_generated.h"
+
+namespace i2cw {
+
+template <class F, int... I>
+__device__ __forceinline__ void static_for_impl(F&& f, std::integer_sequence<int, I...>) {
+  (f(std::integral_constant<int, I>{}), ...);
+}
+template <int N, class F>
+__device__ __forceinline__ void static_for(F&& f) {
+  static_for_impl(f, std::make_integer_sequence<int, N>{});
+}
+
+// sum_j c_j * d[j][e] with compile-time coefficients; zeros skipped, ±1 as add/sub.
+// Only j with (j % JSTEP == JOFF) are included (the pair trick's even/odd halves).
+template <class T, int PT, int JSTEP, int JOFF, int A>
+__device__ __forceinline__ float bt_dot(const float (&d)[A][4], int e) {
+  float acc = 0.f;
+  static_for<A>([&](auto J) {
+    constexpr int j = J;
+    if constexpr (j % JSTEP == JOFF) {
+      constexpr float c = T::BT(PT, j);
+      if constexpr (c == 1.f) acc += d[j][e];
+      else if constexpr (c == -1.f) acc -= d[j][e];
+      else if constexpr (c != 0.f) acc = fmaf(c, d[j][e], acc);
+    }
+  });
+  return acc;
+}
+
+template <int M, int RW, int NT, bool PAIR>
+struct TcCfg {
+  using T = Wino<M, RW>;
+  static constexpr int A = T::alpha;
+  static constexpr int GP = gp_for(A, NT);
+  static constexpr int NS = ns_for(A, NT);
+  static constexpr int NISS = niss_for(GP);
+  static constexpr int NWG = nwg_for(NT);
+  static constexpr int NPASS = A / GP;
+  static constexpr int VCOL = GP * NT;                // first V column in TMEM
+  static constexpr int TMEM_COLS = 512;
+  // one k-step of U in this CTA's shared memory (GP points, hi+lo); a CTA pair splits N
+  static constexpr int UBYTES = GP * 2 * NT * 32 / (PAIR ? 2 : 1);
+  static constexpr int BROWS = PAIR ? NT / 2 : NT;    // B rows (output channels) held per CTA
+  static constexpr int NTHREADS = tc_threads(GP, NT);
+  static constexpr int PPI = GP / NISS;               // points per issuer
+  static_assert(A % GP == 0 && GP % 2 == 0, "passes must hold whole ± pairs");
+  static_assert(NS >= 2 && NS % NWG == 0, "stage ring");
+  static_assert(GP * NT + NS * GP * 16 <= TMEM_COLS, "TMEM budget");
+  static_assert(NT % 16 == 0 && NT >= 16 && NT <= 256, "UMMA N for M=128");
+  static_assert(!PAIR || (NT % 32 == 0 && NT >= 32), "UMMA N for cta_group::2, M=256");
+  static_assert((NT / NWG) % 8 == 0, "epilogue column split");
+  static_assert(GP % NISS == 0, "issuer split");
+};
+
+// PAIR = true: a cluster of 2 CTAs on an SM pair runs tcgen05.mma.cta_group::2 with
+// M = 256 (each CTA's 128 tiles) and N = NT; each CTA stages only its half of the U rows
+// (BROWS = NT/2 output channels), halving the U fill and the B-operand reads per SM. The
+// leader (rank 0) issues all MMAs; the peer's "relay" thread forwards "my V stage and U
+// half are in place" with one remote mbarrier arrive per k-step, and its epilogue's "D
+// read" with one per pass. Commits are multicast to the barriers of both CTAs.
+template <int M, int RW, int NT, bool PAIR>
+__global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
+    fused_tc_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__ CUtensorMap ymap,
+                    const __grid_constant__ Plan pl, const float* __restrict__ u) {
+  using Cfg = TcCfg<M, RW, NT, PAIR>;
+  using T = typename Cfg::T;
+  constexpr int A = Cfg::A, GP = Cfg::GP, NS = Cfg::NS, NISS = Cfg::NISS, NWG = Cfg::NWG;
+  constexpr int NPASS = Cfg::NPASS, VCOL = Cfg::VCOL, PPI = Cfg::PPI, BROWS = Cfg::BROWS;
+  const int NIS = pl.NIS;  // input stages (runtime: fills the shared-memory budget)
+  constexpr uint32_t UBYTES = Cfg::UBYTES;
+  const uint32_t rank = PAIR ? cluster_ctarank() : 0u;  // 0 = MMA leader
+
+  // k-step V slots in TMEM and their grouping into super-stages of KPS k-steps: one
+  // full/empty barrier pair and one U slot per super-stage, so the MMA issuers pay one
+  // wait + commit per KPS k-steps (measured: ~400 cycles of barrier work per k-step with
+  // KPS = 1, above the 384 cycles of UMMA work of a 4-point, N=64 k-step).
+  constexpr int NSLOT = NS;                       // V slots (one per warpgroup)
+  constexpr int KPS = NSLOT >= 4 ? 2 : 1;         // k-steps per super-stage
+  constexpr int NSS = NSLOT / KPS;                // super-stages
+  static_assert(NSLOT % NWG == 0 && NSLOT == NWG, "one V slot per warpgroup");
+
+  extern __shared__ __align__(1024) uint8_t smem[];
+  const uint32_t inplane = (uint32_t)pl.PLANE;  // plane stride (128-aligned)
+  const int NUS = pl.NUS;                         // U super-slots (runtime: SMEM budget)
+  constexpr uint32_t USBYTES = KPS * UBYTES;      // one U super-slot
+  uint8_t* u_smem = smem;                                        // [NUS][USBYTES]        (1024-aligned)
+  uint8_t* o_smem = u_smem + (size_t)NUS * USBYTES;              // [NWG][NOB][OSTRIDE]   (1024-aligned)
+  uint8_t* in_smem = o_smem + (size_t)NWG * pl.NOB * pl.OSTRIDE;  // [NIS][2 planes][PLANE]
+  uint64_t* bars = reinterpret_cast<uint64_t*>(in_smem + (size_t)NIS * 2 * inplane);
+  uint64_t* in_full = bars;             // [NIS]
+  uint64_t* in_empty = in_full + NIS;   // [NIS]
+  uint64_t* st_full = in_empty + NIS;   // [NSS]
+  uint64_t* st_empty = st_full + NSS;   // [NSS]
+  uint64_t* r_full = st_empty + NSS;    // [NSS]  (pair leader: the peer's super-stage relayed)
+  uint64_t* d_full = r_full + NSS;      // [1]
+  uint64_t* d_empty = d_full + 1;       // [1]
+  uint64_t* u_full = d_empty + 1;       // [NUS]
+  uint64_t* u_empty = u_full + NUS;     // [NUS]
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(u_empty + NUS);
+
+  const int warp = threadIdx.x / 32, lane32 = threadIdx.x % 32;
+  int tb, nb;
+  if constexpr (PAIR) {  // clusters of 2 along x: both CTAs share nb, take consecutive tile blocks
+    const int pr = blockIdx.x >> 1;
+    nb = pr % pl.NB;
+    tb = 2 * (pr / pl.NB) + (int)rank;
+  } else {
+    nb = blockIdx.x % pl.NB;
+    tb = blockIdx.x / pl.NB;
+  }
+  const bool cta_active = tb < pl.tile_blocks;  // odd tile-block count: the last peer only helps the MMA
+  const int seg = tb % pl.SEGS;
+  const int tbr = tb / pl.SEGS;
+  const int rb = tbr % pl.PB;
+  const int n = tbr / pl.PB;
+  const int p0 = rb * pl.ROWS;
+  // Channel-chunk rotation: CTA b walks the chunks starting at crot(b), so SMs do not all
+  // stream the same U image at the same time. Both CTAs of a pair rotate alike (their MMAs
+  // consume the same k-step). Each CTA's summation order is fixed: results stay
+  // run-to-run deterministic.
+  const int crot = (int)(((blockIdx.x >> (PAIR ? 1 : 0)) * 5u) % (unsigned)pl.NCC);
+  const int NKS = pl.NKS;
+  const int NKSP = (NKS + KPS - 1) / KPS * KPS;   // k-steps per pass padded to whole super-stages
+  constexpr int PROD_WARP = NWG * 4, UPROD_WARP = NWG * 4 + 1, ISS_WARP0 = NWG * 4 + 2;
+
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < NIS; ++i) { mbar_init(&in_full[i], 1); mbar_init(&in_empty[i], NWG * 128); }
+    for (int i = 0; i < NSS; ++i) {
+      mbar_init(&st_full[i], KPS * 128);  // the KPS warpgroups writing this super-stage
+      mbar_init(&st_empty[i], NISS);
+      mbar_init(&r_full[i], 1);
+    }
+    for (int i = 0; i < NUS; ++i) { mbar_init(&u_full[i], 1); mbar_init(&u_empty[i], NISS); }
+    mbar_init(d_full, NISS);
+    mbar_init(d_empty, NWG * 128 + (PAIR && rank == 0 ? 1 : 0));
+    fence_mbar_init();
+  }
+  if (warp == ISS_WARP0) {  // the first issuer warp owns the TMEM allocation
+    if constexpr (PAIR) { tmem_alloc2(tmem_slot, Cfg::TMEM_COLS); tmem_relinquish2(); }
+    else { tmem_alloc(tmem_slot, Cfg::TMEM_COLS); tmem_relinquish(); }
+  }
+  tc_fence_before();
+  if constexpr (PAIR) cluster_sync_all();
+  else __syncthreads();
+  tc_fence_after();
+  const uint32_t tbase = *tmem_slot;
+
+  if (warp < NWG * 4) {
+    // ===================== transform + epilogue warpgroups =====================
+    const int g = warp / 4;           // == its V slot (NSLOT == NWG)
+    const int l = threadIdx.x % 128;  // TMEM lane == tile slot
+    const int row_l = pl.lane_row[l], tw_l = pl.lane_tw[l];
+    const bool has_slot = row_l != 0xFF;
+    const int col0 = has_slot ? tw_l * M : 0;
+    const uint32_t lane_addr = tbase + ((uint32_t)(l & ~31) << 16);
+    const uint32_t vbase = lane_addr + VCOL + g * GP * 16;
+    const int TSM = pl.TS * M;  // output columns per CTA row segment
+    float* ostage = reinterpret_cast<float*>(o_smem + (size_t)g * pl.NOB * pl.OSTRIDE);
+    // staged row of this tile in the output box (box order: channels, tiles, rows) and its
+    // TMA swizzle: 128B rows (CPW = 32) XOR chunk with r & 7; 64B rows (CPW = 16) with (r>>1) & 3
+    constexpr int CPW = NT / NWG;
+    const int orow = has_slot ? row_l * pl.TS + tw_l : 0;
+    const int oswz = CPW == 32 ? (orow & 7) : ((orow >> 1) & 3);
+    // wait until this warpgroup's V slot may be overwritten (k-step kg's super-stage freed)
+    auto wait_slot = [&](int kg) {
+      const int sg = kg / KPS, use = sg / NSS;
+      if (use > 0) mbar_wait_cluster(&st_empty[sg % NSS], (use - 1) & 1);  // tcgen05.commit
+    };
+
+    int ist = 0, iph = 0;  // input ring slot / phase (incremental: no runtime division)
+    static_for<NPASS>([&](auto PASS_) {
+      constexpr int PASS = PASS_;
+      for (int cc = 0; cc < pl.NCC; ++cc) {
+        const int li = PASS * pl.NCC + cc;
+        if (l == 0) trace_rec(pl.trace, 19 + g, li);
+        mbar_wait(&in_full[ist], iph);
+        if (l == 0) trace_rec(pl.trace, 23 + g, li);
+        const float4* planes = reinterpret_cast<const float4*>(in_smem + (size_t)ist * 2 * inplane);
+        for (int fh = 0; fh < pl.R; ++fh) {
+          const int kg = PASS * NKSP + cc * pl.R + fh;  // global k-step index (padded passes)
+          if (kg % NWG != g) continue;
+          if (l == 0) trace_rec(pl.trace, 0 + g, kg / NWG);
+          wait_slot(kg);
+          tc_fence_after();
+          if (l == 0) trace_rec(pl.trace, 4 + g, kg / NWG);
+          const int off = (has_slot ? (row_l + fh) : 0) * pl.WBOX + col0;
+          if (pl.ablate & 1) {  // DEBUG timing ablation: V = 0 without loads or math
+#pragma unroll
+            for (int c = 0; c < GP * 4; ++c) tmem_st_x4(vbase + c * 4, 0.f, 0.f, 0.f, 0.f);
+          } else {
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+              const float4* src = planes + (size_t)h * (inplane / 16) + off;
+              float d[A][4];
+#pragma unroll
+              for (int j = 0; j < A; ++j) {
+                float4 v = has_slot ? src[j] : make_float4(0.f, 0.f, 0.f, 0.f);
+                d[j][0] = v.x; d[j][1] = v.y; d[j][2] = v.z; d[j][3] = v.w;
+              }
+              static_for<GP / 2>([&](auto Q_) {
+                constexpr int idx0 = PASS * GP + 2 * (int)Q_;  // internal index of this pair slot
+                constexpr int tl0 = 2 * (int)Q_;
+                float va[4], vb[4];
+                if constexpr (idx0 == 0) {  // singles: point 0 and point alpha-1
+#pragma unroll
+                  for (int e = 0; e < 4; ++e) {
+                    va[e] = bt_dot<T, 0, 1, 0>(d, e);
+                    vb[e] = bt_dot<T, A - 1, 1, 0>(d, e);
+                  }
+                } else {  // ± pair (a, a+1): E over even j, O over odd j
+                  constexpr int pa = point_of(idx0, A);
+#pragma unroll
+                  for (int e = 0; e < 4; ++e) {
+                    const float E = bt_dot<T, pa, 2, 0>(d, e);
+                    const float O = bt_dot<T, pa, 2, 1>(d, e);
+                    va[e] = E + O;
+                    vb[e] = E - O;
+                  }
+                }
+                float ha[4], la[4], hb[4], lb[4];
+#pragma unroll
+                for (int e = 0; e < 4; ++e) {
+                  split_tf32(va[e], ha[e], la[e]);
+                  split_tf32(vb[e], hb[e], lb[e]);
+                }
+                const uint32_t ca = vbase + tl0 * 16 + h * 4, cb = ca + 16;
+                tmem_st_x4(ca, ha[0], ha[1], ha[2], ha[3]);
+                tmem_st_x4(ca + 8, la[0], la[1], la[2], la[3]);
+                tmem_st_x4(cb, hb[0], hb[1], hb[2], hb[3]);
+                tmem_st_x4(cb + 8, lb[0], lb[1], lb[2], lb[3]);
+              });
+            }
+          }
+          tmem_wait_st();
+          tc_fence_before();
+          mbar_arrive(&st_full[(kg / KPS) % NSS]);
+          if (l == 0) trace_rec(pl.trace, 8 + g, kg / NWG);
+        }
+        mbar_arrive(&in_empty[ist]);
+        if (++ist == NIS) { ist = 0; iph ^= 1; }
+      }
+      // padding k-steps of the last super-stage (NKS not a multiple of KPS): no V, but the
+      // owning warpgroup still takes its turn so the super-stage's arrival count is met
+      for (int kl = NKS; kl < NKSP; ++kl) {
+        const int kg = PASS * NKSP + kl;
+        if (kg % NWG != g) continue;
+        wait_slot(kg);
+        tc_fence_before();
+        mbar_arrive(&st_full[(kg / KPS) % NSS]);
+      }
+      // ---------- epilogue of this pass: y (+)= A^T M via shared memory + TMA ----------
+      if (l == 0 && g == 0) trace_rec(pl.trace, 27, 2 * PASS);
+      mbar_wait_cluster(d_full, PASS & 1);  // completed by tcgen05.commit
+      tc_fence_after();
+      if (l == 0 && g == 0) trace_rec(pl.trace, 27, 2 * PASS + 1);
+      // One output column i at a time over this warpgroup's CPW channels: every tile's
+      // y[q0 + i][cbase .. cbase+CPW) is one 128-byte (64-byte) row of the staging box,
+      // and the TMA store walks Q with element stride m (positions q0 + i of all tiles).
+      const int qbase = seg * TSM;
+      const int cbase = g * CPW;
+      if (pl.ablate & 4) {  // DEBUG timing ablation: release the accumulators, no y
+        tc_fence_before();
+        mbar_arrive(d_empty);
+      } else {
+        static_for<M>([&](auto I_) {
+          constexpr int i = I_;
+          // staging buffer reuse: the TMA store that last read it must be done reading
+          const int ob = i % pl.NOB;
+          if (l == 0) {
+            if (pl.NOB == 2) bulk_wait_group_read<1>();
+            else bulk_wait_group_read<0>();
+          }
+          named_bar_sync(1 + g, 128);
+          float4* stg = reinterpret_cast<float4*>(ostage + (size_t)ob * (pl.OSTRIDE / 4)) + (size_t)orow * (CPW / 4);
+#pragma unroll 1
+          for (int hh = 0; hh < CPW / 16; ++hh) {  // 16 channels at a time (register budget)
+            float o[16];
+#pragma unroll
+            for (int e = 0; e < 16; ++e) o[e] = 0.f;
+            static_for<GP / 2>([&](auto Q_) {
+              constexpr int idx0 = PASS * GP + 2 * (int)Q_;  // pair slot (internal points idx0, idx0+1)
+              constexpr int tl0 = 2 * (int)Q_;
+              float ma[16], mb[16];
+              tmem_ld_x16(lane_addr + tl0 * NT + cbase + 16 * hh, ma);
+              tmem_ld_x16(lane_addr + (tl0 + 1) * NT + cbase + 16 * hh, mb);
+              tmem_wait_ld();
+              if constexpr (idx0 == 0) {
+                constexpr float c0 = T::AT(i, 0), c1 = T::AT(i, A - 1);
+#pragma unroll
+                for (int e = 0; e < 16; ++e) {
+                  if constexpr (c0 != 0.f) o[e] = fmaf(c0, ma[e], o[e]);
+                  if constexpr (c1 != 0.f) o[e] = fmaf(c1, mb[e], o[e]);
+                }
+              } else {  // AT[i][a+1] = (-1)^i AT[i][a] (pair structure)
+                constexpr int pa = point_of(idx0, A);
+                constexpr float ca = T::AT(i, pa);
+#pragma unroll
+                for (int e = 0; e < 16; ++e) {
+                  const float sv = (i % 2 == 0) ? (ma[e] + mb[e]) : (ma[e] - mb[e]);
+                  if constexpr (ca == 1.f) o[e] += sv;
+                  else if constexpr (ca != 0.f) o[e] = fmaf(ca, sv, o[e]);
+                }
+              }
+            });
+            if (has_slot) {
+#pragma unroll
+              for (int j = 0; j < 4; ++j)
+                stg[(4 * hh + j) ^ oswz] = make_float4(o[4 * j], o[4 * j + 1], o[4 * j + 2], o[4 * j + 3]);
+            }
+          }
+          if constexpr (i == M - 1) {  // accumulators fully read: the issuers may start the next pass
+            tc_fence_before();
+            mbar_arrive(d_empty);
+          }
+          fence_proxy_async_smem();
+          named_bar_sync(1 + g, 128);
+          if (l == 0) {
+            const float* box = ostage + (size_t)ob * (pl.OSTRIDE / 4);
+            const int k0 = nb * NT + cbase;
+            if (cta_active) {
+              if constexpr (PASS == 0) tma_store_4d(&ymap, box, k0, qbase + i, p0, n);
+              else tma_reduce_add_4d(&ymap, box, k0, qbase + i, p0, n);
+            }
+            bulk_commit_group();
+          }
+        });
+      }
+      // this pass's writes must be complete before the next pass's reduce-add
+      if (l == 0) bulk_wait_group_all();
+      if (l == 0 && g == 0) trace_rec(pl.trace, 28, PASS);
+    });
+  } else if (warp == PROD_WARP) {
+    // ====================== input-row TMA producer ======================
+    if (lane32 == 0) {
+      tma_prefetch_desc(&xmap);
+      tma_prefetch_desc(&ymap);
+      const int wstart = seg * pl.TS * M - pl.pad_w;
+      const int hstart = p0 - pl.pad_h;
+      int ist = 0, iph = 0, first = 1;  // slot, round parity, still in the first round
+      for (int pass = 0; pass < NPASS; ++pass) {
+        for (int cc = 0; cc < pl.NCC; ++cc) {
+          if (!first) mbar_wait(&in_empty[ist], iph ^ 1);
+          uint8_t* dst = in_smem + (size_t)ist * 2 * inplane;
+          const int ca = cc + crot < pl.NCC ? cc + crot : cc + crot - pl.NCC;  // actual chunk
+          if (pl.ablate & 16) {  // DEBUG timing ablation: no input rows (stage reused as is)
+            mbar_arrive(&in_full[ist]);
+          } else {
+            mbar_expect_tx(&in_full[ist], 2u * (uint32_t)pl.BOXB);
+            tma_load_4d(dst, &xmap, &in_full[ist], ca * 8, wstart, hstart, n);
+            tma_load_4d(dst + inplane, &xmap, &in_full[ist], ca * 8 + 4, wstart, hstart, n);
+          }
+          if (++ist == NIS) { ist = 0; iph ^= 1; first = 0; }
+        }
+      }
+    }
+    __syncwarp();
+  } else if (warp == UPROD_WARP) {
+    // ================= U (transformed filter) super-slot ring =================
+    if (lane32 == 0) {
+      const size_t kstride = (size_t)A * 2 * NT * 8;  // floats per k-step (both layouts)
+      int us = 0, uph = 0, first = 1;
+      for (int pass = 0; pass < NPASS; ++pass) {
+        // this CTA's B rows of the pass's GP points, hi+lo, contiguous (pair: its N half)
+        const float* src0 = u + (PAIR ? u_offset_pair(NT, A, nb, NKS, 0, (int)rank, pass * GP)
+                                      : u_offset(NT, A, nb, NKS, 0, pass * GP, 0));
+        for (int kl0 = 0; kl0 < NKSP; kl0 += KPS) {
+          trace_rec(pl.trace, 30, pass * NKSP + kl0);
+          if (!first) mbar_wait_cluster(&u_empty[us], uph ^ 1);  // completed by tcgen05.commit
+          trace_rec(pl.trace, 31, pass * NKSP + kl0);
+          const int nreal = NKS - kl0 < KPS ? NKS - kl0 : KPS;
+          const uint32_t ub = (pl.ablate & 8) ? 1024u : UBYTES;  // DEBUG timing ablation: shrink
+          mbar_expect_tx(&u_full[us], (uint32_t)nreal * ub);
+          for (int pos = 0; pos < nreal; ++pos) {
+            const int kl = kl0 + pos, cc = kl / pl.R, fh = kl - cc * pl.R;
+            const int ca = cc + crot < pl.NCC ? cc + crot : cc + crot - pl.NCC;
+            bulk_load(u_smem + (size_t)us * USBYTES + (size_t)pos * UBYTES, src0 + (size_t)(ca * pl.R + fh) * kstride,
+                      ub, &u_full[us]);
+          }
+          if (++us == NUS) { us = 0; uph ^= 1; first = 0; }
+        }
+      }
+    }
+    __syncwarp();
+  } else {
+    // ============================= MMA issuers =============================
+    const int iss = warp - ISS_WARP0;  // owns points tl = iss * PPI .. iss * PPI + PPI - 1
+    if (lane32 == 0 && rank == 0) {
+      constexpr uint32_t idesc = idesc_tf32(PAIR ? 256 : 128, NT);
+      // descriptor of U super-slot 0, k-step 0, point 0, hi; other images = + (byte offset >> 4)
+      const uint64_t bdesc0 = umma_desc_kmajor_noswizzle(smem_u32(u_smem), BROWS * 16, 128);
+      int ss = 0, sph = 0, us = 0, uph = 0;  // super-stage / U super-slot and their round parities
+      int sgi = 0;
+      for (int pass = 0; pass < NPASS; ++pass) {
+        if (pass > 0) {
+          mbar_wait_cluster(d_empty, (pass - 1) & 1);
+          tc_fence_after();
+        }
+        for (int kl0 = 0; kl0 < NKSP; kl0 += KPS, ++sgi) {
+          if (iss == 0) trace_rec(pl.trace, 29, sgi);
+          mbar_wait(&st_full[ss], sph);
+          mbar_wait(&u_full[us], uph);
+          if constexpr (PAIR) mbar_wait_cluster(&r_full[ss], sph);  // the peer's V + U half
+          tc_fence_after();
+          if (iss == 0) trace_rec(pl.trace, 16, sgi);
+          if (!(pl.ablate & 2)) {  // DEBUG timing ablation: skip the MMAs (commits still signal)
+#pragma unroll
+            for (int pos = 0; pos < KPS; ++pos) {
+              const int kl = kl0 + pos;
+              if (kl >= NKS) break;
+              const uint64_t bk = bdesc0 + (uint64_t)((us * USBYTES + pos * UBYTES) >> 4);
+              const uint32_t va = tbase + VCOL + (ss * KPS + pos) * GP * 16;
+              // product order lo*hi, hi*lo, hi*hi (small terms first), points innermost
+#pragma unroll
+              for (int prod = 0; prod < 3; ++prod) {
+#pragma unroll
+                for (int pi = 0; pi < PPI; ++pi) {
+                  const int tl = iss * PPI + pi;
+                  const uint32_t a = va + tl * 16 + (prod == 0 ? 8 : 0);
+                  const uint64_t bd = bk + (uint64_t)(((tl * 2 + (prod == 1 ? 1 : 0)) * BROWS * 32) >> 4);
+                  const uint32_t acc = (kl > 0 || prod > 0) ? 1u : 0u;
+                  if constexpr (PAIR) mma2_tf32_ts(tbase + tl * NT, a, bd, idesc, acc);
+                  else mma_tf32_ts(tbase + tl * NT, a, bd, idesc, acc);
+                }
+              }
+            }
+          }
+          if (iss == 0) trace_rec(pl.trace, 17, sgi);
+          if constexpr (PAIR) { mma_commit2(&st_empty[ss]); mma_commit2(&u_empty[us]); }
+          else { mma_commit(&st_empty[ss]); mma_commit(&u_empty[us]); }
+          if (iss == 0) trace_rec(pl.trace, 18, sgi);
+          if (++ss == NSS) { ss = 0; sph ^= 1; }
+          if (++us == NUS) { us = 0; uph ^= 1; }
+        }
+        if constexpr (PAIR) mma_commit2(d_full);
+        else mma_commit(d_full);
+      }
+    } else if (PAIR && lane32 == 0 && rank == 1 && iss == 0) {
+      // ===== pair peer relay: forward this CTA's super-stage readiness / D drain =====
+      const uint32_t lead_rfull = mapa_shared(r_full, 0), lead_dempty = mapa_shared(d_empty, 0);
+      int ss = 0, sph = 0, us = 0, uph = 0, sgi = 0;
+      for (int pass = 0; pass < NPASS; ++pass) {
+        for (int kl0 = 0; kl0 < NKSP; kl0 += KPS, ++sgi) {
+          mbar_wait(&st_full[ss], sph);
+          mbar_wait(&u_full[us], uph);
+          tc_fence_after();
+          mbar_arrive_remote(lead_rfull + 8u * ss);
+          trace_rec(pl.trace, 17, sgi);
+          if (++ss == NSS) { ss = 0; sph ^= 1; }
+          if (++us == NUS) { us = 0; uph ^= 1; }
+        }
+        if (pass + 1 < NPASS) {  // this CTA's epilogue has read its D: the leader may overwrite it
+          mbar_wait(d_empty, pass & 1);
+          tc_fence_after();
+          mbar_arrive_remote(lead_dempty);
+        }
+      }
+    }
+    __syncwarp();
+  }
+
+  tc_fence_before();
+  if constexpr (PAIR) cluster_sync_all();
+  else __syncthreads();
+  if (warp == ISS_WARP0) {
+    tc_fence_after();
+    if constexpr (PAIR) tmem_dealloc2(tbase, Cfg::TMEM_COLS);
+    else tmem_dealloc(tbase, Cfg::TMEM_COLS);
+  }
+}
+
+template <int M, int RW, int NT, bool PAIR>
+static cudaError_t launch_tc_t(const CUtensorMap& xmap, const CUtensorMap& ymap, const Plan& pl, const float* u,
+                               cudaStream_t stream) {
+  using Cfg = TcCfg<M, RW, NT, PAIR>;
+  auto kern = fused_tc_kernel<M, RW, NT, PAIR>;
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, pl.smem_bytes);
+  if (e != cudaSuccess) return e;
+  if constexpr (PAIR) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(2 * ((pl.tile_blocks + 1) / 2) * pl.NB);
+    cfg.blockDim = dim3(Cfg::NTHREADS);
+    cfg.dynamicSmemBytes = pl.smem_bytes;
+    cfg.stream = stream;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = 2;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    e = cudaLaunchKernelEx(&cfg, kern, xmap, ymap, pl, u);
+    if (e != cudaSuccess) return e;
+  } else {
+    kern<<<pl.tile_blocks * pl.NB, Cfg::NTHREADS, pl.smem_bytes, stream>>>(xmap, ymap, pl, u);
+  }
+  return cudaGetLastError();
+}
+
+}  // namespace i2cw

@@ -18,17 +18,18 @@ for name in sys.argv[1:] or ["cfg2"]:
     x = torch.rand((N, H, W, C), device="cuda"); w = torch.rand((K, R, S, C), device="cuda")
     P, Q = H + 2 * ph - R + 1, W + 2 * pw - S + 1
     y = torch.empty((N, P, Q, K), device="cuda")
-    tr = torch.zeros(32 * 512, dtype=torch.int64, device="cuda")
+    tr = torch.zeros(2 * 32 * 512, dtype=torch.int64, device="cuda")
     for _ in range(3):
         tr.zero_()
         rc = L.i2cw_debug_trace(0, N, H, W, C, K, R, S, ph, pw, x.data_ptr(), w.data_ptr(), y.data_ptr(), tr.data_ptr(),
                                 torch.cuda.current_stream().cuda_stream)
         assert rc == 0
     torch.cuda.synchronize()
-    t = tr.cpu().numpy().reshape(32, 512).astype(np.int64)
-    t0 = t[t > 0].min()
-    t = np.where(t > 0, t - t0, -1)
-    def v(k): return t[k][t[k] >= 0]
+    T2 = tr.cpu().numpy().reshape(2, 32, 512).astype(np.int64)
+    t0 = T2[T2 > 0].min()
+    T2 = np.where(T2 > 0, T2 - t0, -1)   # ns (globaltimer)
+    t = T2[0]
+    def v(k, cta=0): return T2[cta][k][T2[cta][k] >= 0]
     pl = i2cw.debug_plan(kind, N, H, W, C, K, R, S, ph, pw)
     print(f"== {name}: plan {pl}")
     nwg = 4 if pl["NT"] == 64 else 2
@@ -51,8 +52,22 @@ for name in sys.argv[1:] or ["cfg2"]:
     print("WG0 per-warp arrive minus warp0 (median):", [float(np.median(A_[w] - A_[0])) for w in range(4)])
     print("epilogue d_full wait (before, after):", v(27).tolist(), " end:", v(28).tolist())
     # per k-step critical path sample: ks 8..15
-    print("kg: WG arrive(last warp of WG0 only for g=0) | issuer ready | issued | committed")
+    print("kg: CTA0 WG arrive | CTA1 WG arrive | CTA0 issuer ready | issued | committed   (ns)")
     for kg in range(8, 16):
         g = kg % nwg; i = kg // nwg
-        arrive = v(8 + g)[i] if i < len(v(8 + g)) else None
-        print(f"  {kg:3d} g{g} arrive {arrive}  ready {w16[kg]}  issued {w17[kg]}  commit {w18[kg]}")
+        a0 = v(8 + g, 0)[i] if i < len(v(8 + g, 0)) else None
+        a1 = v(8 + g, 1)[i] if i < len(v(8 + g, 1)) else None
+        print(f"  {kg:3d} g{g} {a0} {a1}  ready {w16[kg]}  issued {w17[kg]}  commit {w18[kg]}")
+    for cta in (0, 1):
+        print(f"CTA{cta} WG0 start/after-wait/arrive first 4:", list(zip(v(0, cta)[:4].tolist(), v(4, cta)[:4].tolist(), v(8, cta)[:4].tolist())),
+              " in_full waits:", list(zip(v(19, cta)[:4].tolist(), v(23, cta)[:4].tolist())))
+    r29, r16, r17 = v(29, 1), v(16, 1), v(17, 1)
+    if len(r29):
+        print("relay (CTA1): kg: after st_full, after u_full, after remote arrive")
+        for kg in range(8, 12):
+            print("   ", kg, r29[kg], r16[kg], r17[kg])
+    u30, u31 = v(30), v(31)
+    if len(u30):
+        print("U producer (CTA0): kg: before u_empty wait, issue time, issuer ready (u_full done)")
+        for kg in range(0, 16):
+            print("   ", kg, u30[kg], u31[kg], w16[kg] if kg < len(w16) else None)
