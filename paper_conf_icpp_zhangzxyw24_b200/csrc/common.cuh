@@ -99,14 +99,24 @@ struct UTag {
 };
 
 #if defined(__CUDACC__)
-// Debug timeline: CTA b < 2, kind k, entry i -> trace[(b * 32 + k) * 512 + i] = globaltimer (ns;
-// comparable across the two SMs of a CTA pair).
-__device__ __forceinline__ void trace_rec(unsigned long long* tr, int kind, int i) {
-  if (tr != nullptr && blockIdx.x < 2 && i < 512) {
+// Debug timeline: CTA b < 2, kind k, entry i -> trace[(b * 32 + k) * 512 + i] = clock64 of the
+// SM (cycles; not comparable across the two SMs of a CTA pair). The "memory" clobber keeps
+// the compiler from moving loads/stores across a trace point.
+// Timeline tracing (tools/trace_run.py) is compiled in only with `make TRACE=1`
+// (-DI2CW_TRACE=1): in the product build trace_rec() is empty and costs no issue slots.
+#ifndef I2CW_TRACE
+#define I2CW_TRACE 0
+#endif
+__device__ __forceinline__ void trace_rec(unsigned long long* tr, int kind, int i, bool on = true) {
+#if I2CW_TRACE
+  if (on && tr != nullptr && blockIdx.x < 2 && i < 512) {
     unsigned long long t;
-    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    asm volatile("mov.u64 %0, %%clock64;" : "=l"(t)::"memory");
     tr[(blockIdx.x * 32 + kind) * 512 + i] = t;
   }
+#else
+  (void)tr; (void)kind; (void)i; (void)on;
+#endif
 }
 // ----------------------------------------------------------------------------
 // PTX helpers
@@ -249,6 +259,15 @@ __device__ __forceinline__ void mbar_wait_cluster(uint64_t* bar, uint32_t parity
   while (!mbar_try_wait_cluster(bar, parity)) {
     if (globaltimer() - t0 > 4000000000ull) __trap();
   }
+}
+
+// Wait on a barrier completed by tcgen05.commit: CTA-scope acquire for a lone CTA (the
+// cluster-scope form compiles to an L1 invalidate, CCTL.IVALL, on every successful wait),
+// cluster scope when the commit comes from the CTA pair's leader.
+template <bool CLUSTER>
+__device__ __forceinline__ void mbar_wait_tc(uint64_t* bar, uint32_t parity) {
+  if constexpr (CLUSTER) mbar_wait_cluster(bar, parity);
+  else mbar_wait(bar, parity);
 }
 
 // ---- tcgen05 --------------------------------------------------------------

@@ -68,6 +68,41 @@ __device__ __forceinline__ float bt_dot(const float (&d)[A][4], int e) {
   return acc;
 }
 
+// Packed (sm_100 FFMA2/FADD2/FMUL2) form of bt_dot over one channel pair p: d[j][p] holds
+// channels (2p, 2p+1) of input position j. Halves the FP issue slots of the transform.
+template <class T, int PT, int JSTEP, int JOFF, int A>
+__host__ __device__ constexpr int bt_first_nz() {
+  for (int j = 0; j < A; ++j)
+    if (j % JSTEP == JOFF && T::BT(PT, j) != 0.f) return j;
+  return -1;
+}
+template <class T, int PT, int JSTEP, int JOFF, int A>
+__device__ __forceinline__ float2 bt_dot2(const float2 (&d)[A][2], int p) {
+  constexpr int j0 = bt_first_nz<T, PT, JSTEP, JOFF, A>();
+  if constexpr (j0 < 0) {
+    return make_float2(0.f, 0.f);
+  } else {
+    constexpr float c0 = T::BT(PT, j0);
+    float2 acc = c0 == 1.f ? d[j0][p] : __fmul2_rn(make_float2(c0, c0), d[j0][p]);
+    static_for<A>([&](auto J) {
+      constexpr int j = J;
+      if constexpr (j > j0 && j % JSTEP == JOFF) {
+        constexpr float c = T::BT(PT, j);
+        if constexpr (c == 1.f) acc = __fadd2_rn(acc, d[j][p]);
+        else if constexpr (c != 0.f) acc = __ffma2_rn(make_float2(c, c), d[j][p], acc);
+      }
+    });
+    return acc;
+  }
+}
+// 3xTF32 operand split of a channel pair: hi = v truncated to tf32 (exactly representable,
+// so the tensor core's own fp32->tf32 conversion mode does not matter), lo = v - hi (exact).
+__device__ __forceinline__ void split_tf32x2(float2 v, float2& hi, float2& lo) {
+  hi.x = __uint_as_float(__float_as_uint(v.x) & 0xFFFFE000u);
+  hi.y = __uint_as_float(__float_as_uint(v.y) & 0xFFFFE000u);
+  lo = __ffma2_rn(make_float2(-1.f, -1.f), hi, v);
+}
+
 template <int M, int RW, int NT, bool PAIR>
 struct TcCfg {
   using T = Wino<M, RW>;
@@ -115,10 +150,10 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
   // full/empty barrier pair and one U slot per super-stage, so the MMA issuers pay one
   // wait + commit per KPS k-steps (measured: ~400 cycles of barrier work per k-step with
   // KPS = 1, above the 384 cycles of UMMA work of a 4-point, N=64 k-step).
-  constexpr int NSLOT = NS;                       // V slots (one per warpgroup)
+  constexpr int NSLOT = NS;                       // V slots in TMEM (one per warpgroup)
+  static_assert(NSLOT == NWG && (NWG & (NWG - 1)) == 0, "one V slot per warpgroup, power of 2");
   constexpr int KPS = NSLOT >= 4 ? 2 : 1;         // k-steps per super-stage
   constexpr int NSS = NSLOT / KPS;                // super-stages
-  static_assert(NSLOT % NWG == 0 && NSLOT == NWG, "one V slot per warpgroup");
 
   extern __shared__ __align__(1024) uint8_t smem[];
   const uint32_t inplane = (uint32_t)pl.PLANE;  // plane stride (128-aligned)
@@ -165,15 +200,17 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
   constexpr int PROD_WARP = NWG * 4, UPROD_WARP = NWG * 4 + 1, ISS_WARP0 = NWG * 4 + 2;
 
   if (threadIdx.x == 0) {
-    for (int i = 0; i < NIS; ++i) { mbar_init(&in_full[i], 1); mbar_init(&in_empty[i], NWG * 128); }
+    // transform-warp arrivals are warp-elected (one lane after __syncwarp): 128 or 512
+    // per-thread arrivals on one barrier word serialise in the shared-memory atomic unit
+    for (int i = 0; i < NIS; ++i) { mbar_init(&in_full[i], 1); mbar_init(&in_empty[i], NWG * 4); }
     for (int i = 0; i < NSS; ++i) {
-      mbar_init(&st_full[i], KPS * 128);  // the KPS warpgroups writing this super-stage
+      mbar_init(&st_full[i], KPS * 4);  // the 4 warps of each of the KPS warpgroups of this super-stage
       mbar_init(&st_empty[i], NISS);
       mbar_init(&r_full[i], 1);
     }
     for (int i = 0; i < NUS; ++i) { mbar_init(&u_full[i], 1); mbar_init(&u_empty[i], NISS); }
     mbar_init(d_full, NISS);
-    mbar_init(d_empty, NWG * 128 + (PAIR && rank == 0 ? 1 : 0));
+    mbar_init(d_empty, NWG * 4 + (PAIR && rank == 0 ? 1 : 0));
     fence_mbar_init();
   }
   if (warp == ISS_WARP0) {  // the first issuer warp owns the TMEM allocation
@@ -194,7 +231,6 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
     const bool has_slot = row_l != 0xFF;
     const int col0 = has_slot ? tw_l * M : 0;
     const uint32_t lane_addr = tbase + ((uint32_t)(l & ~31) << 16);
-    const uint32_t vbase = lane_addr + VCOL + g * GP * 16;
     const int TSM = pl.TS * M;  // output columns per CTA row segment
     float* ostage = reinterpret_cast<float*>(o_smem + (size_t)g * pl.NOB * pl.OSTRIDE);
     // staged row of this tile in the output box (box order: channels, tiles, rows) and its
@@ -202,98 +238,100 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
     constexpr int CPW = NT / NWG;
     const int orow = has_slot ? row_l * pl.TS + tw_l : 0;
     const int oswz = CPW == 32 ? (orow & 7) : ((orow >> 1) & 3);
-    // wait until this warpgroup's V slot may be overwritten (k-step kg's super-stage freed)
-    auto wait_slot = [&](int kg) {
+    // Warpgroup g owns V slot g and computes the k-steps kg = g (mod NWG) of every pass
+    // (kg = PASS * NKSP + cc * R + fh): the four warpgroups' transforms interleave on the
+    // SMSPs, each k-step's full V (GP points x 8 channels, hi + lo) written by one warpgroup.
+    const uint32_t vbase = lane_addr + VCOL + g * GP * 16;
+    auto wait_slot = [&](int kg) {  // this slot's previous k-step consumed (tcgen05.commit)
       const int sg = kg / KPS, use = sg / NSS;
-      if (use > 0) mbar_wait_cluster(&st_empty[sg % NSS], (use - 1) & 1);  // tcgen05.commit
+      if (use > 0) mbar_wait_tc<PAIR>(&st_empty[sg % NSS], (use - 1) & 1);
     };
-
     int ist = 0, iph = 0;  // input ring slot / phase (incremental: no runtime division)
     static_for<NPASS>([&](auto PASS_) {
       constexpr int PASS = PASS_;
       for (int cc = 0; cc < pl.NCC; ++cc) {
-        const int li = PASS * pl.NCC + cc;
-        if (l == 0) trace_rec(pl.trace, 19 + g, li);
+        const int kb = PASS * NKSP + cc * pl.R;  // first k-step of this chunk
+        trace_rec(pl.trace, 19 + g, PASS * pl.NCC + cc, l == 0);
+        // every warpgroup waits for every chunk (also one it has no k-step in, R < NWG) so
+        // its in_empty arrival can never run ahead into the slot's next phase
         mbar_wait(&in_full[ist], iph);
-        if (l == 0) trace_rec(pl.trace, 23 + g, li);
+        trace_rec(pl.trace, 23 + g, PASS * pl.NCC + cc, l == 0);
         const float4* planes = reinterpret_cast<const float4*>(in_smem + (size_t)ist * 2 * inplane);
-        for (int fh = 0; fh < pl.R; ++fh) {
-          const int kg = PASS * NKSP + cc * pl.R + fh;  // global k-step index (padded passes)
-          if (kg % NWG != g) continue;
-          if (l == 0) trace_rec(pl.trace, 0 + g, kg / NWG);
+        for (int fh = (g - kb) & (NWG - 1); fh < pl.R; fh += NWG) {
+          const int kg = kb + fh;
+          trace_rec(pl.trace, 0 + g, kg / NWG, l == 0);
           wait_slot(kg);
           tc_fence_after();
-          if (l == 0) trace_rec(pl.trace, 4 + g, kg / NWG);
-          const int off = (has_slot ? (row_l + fh) : 0) * pl.WBOX + col0;
+          trace_rec(pl.trace, 4 + g, kg / NWG, l == 0);
           if (pl.ablate & 1) {  // DEBUG timing ablation: V = 0 without loads or math
 #pragma unroll
             for (int c = 0; c < GP * 4; ++c) tmem_st_x4(vbase + c * 4, 0.f, 0.f, 0.f, 0.f);
           } else {
+            const int off = (has_slot ? (row_l + fh) : 0) * pl.WBOX + col0;
 #pragma unroll
-            for (int h = 0; h < 2; ++h) {
+            for (int h = 0; h < 2; ++h) {  // channel quads (input planes)
               const float4* src = planes + (size_t)h * (inplane / 16) + off;
-              float d[A][4];
+              float2 d[A][2];
 #pragma unroll
               for (int j = 0; j < A; ++j) {
-                float4 v = has_slot ? src[j] : make_float4(0.f, 0.f, 0.f, 0.f);
-                d[j][0] = v.x; d[j][1] = v.y; d[j][2] = v.z; d[j][3] = v.w;
+                const float4 v = has_slot ? src[j] : make_float4(0.f, 0.f, 0.f, 0.f);
+                d[j][0] = make_float2(v.x, v.y);
+                d[j][1] = make_float2(v.z, v.w);
               }
               static_for<GP / 2>([&](auto Q_) {
                 constexpr int idx0 = PASS * GP + 2 * (int)Q_;  // internal index of this pair slot
                 constexpr int tl0 = 2 * (int)Q_;
-                float va[4], vb[4];
-                if constexpr (idx0 == 0) {  // singles: point 0 and point alpha-1
+                float2 ha[2], la[2], hb[2], lb[2];
 #pragma unroll
-                  for (int e = 0; e < 4; ++e) {
-                    va[e] = bt_dot<T, 0, 1, 0>(d, e);
-                    vb[e] = bt_dot<T, A - 1, 1, 0>(d, e);
+                for (int p = 0; p < 2; ++p) {
+                  float2 va, vb;
+                  if constexpr (idx0 == 0) {  // singles: point 0 and point alpha-1
+                    va = bt_dot2<T, 0, 1, 0>(d, p);
+                    vb = bt_dot2<T, A - 1, 1, 0>(d, p);
+                  } else {  // ± pair (a, a+1): E over even j, O over odd j
+                    constexpr int pa = point_of(idx0, A);
+                    const float2 E = bt_dot2<T, pa, 2, 0>(d, p);
+                    const float2 O = bt_dot2<T, pa, 2, 1>(d, p);
+                    va = __fadd2_rn(E, O);
+                    vb = __ffma2_rn(make_float2(-1.f, -1.f), O, E);
                   }
-                } else {  // ± pair (a, a+1): E over even j, O over odd j
-                  constexpr int pa = point_of(idx0, A);
-#pragma unroll
-                  for (int e = 0; e < 4; ++e) {
-                    const float E = bt_dot<T, pa, 2, 0>(d, e);
-                    const float O = bt_dot<T, pa, 2, 1>(d, e);
-                    va[e] = E + O;
-                    vb[e] = E - O;
-                  }
-                }
-                float ha[4], la[4], hb[4], lb[4];
-#pragma unroll
-                for (int e = 0; e < 4; ++e) {
-                  split_tf32(va[e], ha[e], la[e]);
-                  split_tf32(vb[e], hb[e], lb[e]);
+                  split_tf32x2(va, ha[p], la[p]);
+                  split_tf32x2(vb, hb[p], lb[p]);
                 }
                 const uint32_t ca = vbase + tl0 * 16 + h * 4, cb = ca + 16;
-                tmem_st_x4(ca, ha[0], ha[1], ha[2], ha[3]);
-                tmem_st_x4(ca + 8, la[0], la[1], la[2], la[3]);
-                tmem_st_x4(cb, hb[0], hb[1], hb[2], hb[3]);
-                tmem_st_x4(cb + 8, lb[0], lb[1], lb[2], lb[3]);
+                tmem_st_x4(ca, ha[0].x, ha[0].y, ha[1].x, ha[1].y);
+                tmem_st_x4(ca + 8, la[0].x, la[0].y, la[1].x, la[1].y);
+                tmem_st_x4(cb, hb[0].x, hb[0].y, hb[1].x, hb[1].y);
+                tmem_st_x4(cb + 8, lb[0].x, lb[0].y, lb[1].x, lb[1].y);
               });
             }
           }
+          trace_rec(pl.trace, 12 + g, kg / NWG, l == 0);
           tmem_wait_st();
           tc_fence_before();
-          mbar_arrive(&st_full[(kg / KPS) % NSS]);
-          if (l == 0) trace_rec(pl.trace, 8 + g, kg / NWG);
+          __syncwarp();
+          if (lane32 == 0) mbar_arrive(&st_full[(kg / KPS) % NSS]);
+          trace_rec(pl.trace, 8 + g, kg / NWG, l == 0);
         }
-        mbar_arrive(&in_empty[ist]);
+        __syncwarp();
+        if (lane32 == 0) mbar_arrive(&in_empty[ist]);
         if (++ist == NIS) { ist = 0; iph ^= 1; }
       }
       // padding k-steps of the last super-stage (NKS not a multiple of KPS): no V, but the
       // owning warpgroup still takes its turn so the super-stage's arrival count is met
       for (int kl = NKS; kl < NKSP; ++kl) {
         const int kg = PASS * NKSP + kl;
-        if (kg % NWG != g) continue;
+        if ((kg & (NWG - 1)) != g) continue;
         wait_slot(kg);
         tc_fence_before();
-        mbar_arrive(&st_full[(kg / KPS) % NSS]);
+        __syncwarp();
+        if (lane32 == 0) mbar_arrive(&st_full[(kg / KPS) % NSS]);
       }
       // ---------- epilogue of this pass: y (+)= A^T M via shared memory + TMA ----------
-      if (l == 0 && g == 0) trace_rec(pl.trace, 27, 2 * PASS);
-      mbar_wait_cluster(d_full, PASS & 1);  // completed by tcgen05.commit
+      trace_rec(pl.trace, 27, 2 * PASS, l == 0 && g == 0);
+      mbar_wait_tc<PAIR>(d_full, PASS & 1);  // completed by tcgen05.commit
       tc_fence_after();
-      if (l == 0 && g == 0) trace_rec(pl.trace, 27, 2 * PASS + 1);
+      trace_rec(pl.trace, 27, 2 * PASS + 1, l == 0 && g == 0);
       // One output column i at a time over this warpgroup's CPW channels: every tile's
       // y[q0 + i][cbase .. cbase+CPW) is one 128-byte (64-byte) row of the staging box,
       // and the TMA store walks Q with element stride m (positions q0 + i of all tiles).
@@ -301,7 +339,8 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
       const int cbase = g * CPW;
       if (pl.ablate & 4) {  // DEBUG timing ablation: release the accumulators, no y
         tc_fence_before();
-        mbar_arrive(d_empty);
+        __syncwarp();
+        if (lane32 == 0) mbar_arrive(d_empty);
       } else {
         static_for<M>([&](auto I_) {
           constexpr int i = I_;
@@ -351,7 +390,8 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
           }
           if constexpr (i == M - 1) {  // accumulators fully read: the issuers may start the next pass
             tc_fence_before();
-            mbar_arrive(d_empty);
+            __syncwarp();
+            if (lane32 == 0) mbar_arrive(d_empty);
           }
           fence_proxy_async_smem();
           named_bar_sync(1 + g, 128);
@@ -368,7 +408,7 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
       }
       // this pass's writes must be complete before the next pass's reduce-add
       if (l == 0) bulk_wait_group_all();
-      if (l == 0 && g == 0) trace_rec(pl.trace, 28, PASS);
+      trace_rec(pl.trace, 28, PASS, l == 0 && g == 0);
     });
   } else if (warp == PROD_WARP) {
     // ====================== input-row TMA producer ======================
@@ -406,7 +446,7 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
                                       : u_offset(NT, A, nb, NKS, 0, pass * GP, 0));
         for (int kl0 = 0; kl0 < NKSP; kl0 += KPS) {
           trace_rec(pl.trace, 30, pass * NKSP + kl0);
-          if (!first) mbar_wait_cluster(&u_empty[us], uph ^ 1);  // completed by tcgen05.commit
+          if (!first) mbar_wait_tc<PAIR>(&u_empty[us], uph ^ 1);  // completed by tcgen05.commit
           trace_rec(pl.trace, 31, pass * NKSP + kl0);
           const int nreal = NKS - kl0 < KPS ? NKS - kl0 : KPS;
           const uint32_t ub = (pl.ablate & 8) ? 1024u : UBYTES;  // DEBUG timing ablation: shrink
@@ -433,16 +473,16 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
       int sgi = 0;
       for (int pass = 0; pass < NPASS; ++pass) {
         if (pass > 0) {
-          mbar_wait_cluster(d_empty, (pass - 1) & 1);
+          mbar_wait_tc<PAIR>(d_empty, (pass - 1) & 1);
           tc_fence_after();
         }
         for (int kl0 = 0; kl0 < NKSP; kl0 += KPS, ++sgi) {
-          if (iss == 0) trace_rec(pl.trace, 29, sgi);
+          trace_rec(pl.trace, 29, sgi, iss == 0);
           mbar_wait(&st_full[ss], sph);
           mbar_wait(&u_full[us], uph);
           if constexpr (PAIR) mbar_wait_cluster(&r_full[ss], sph);  // the peer's V + U half
           tc_fence_after();
-          if (iss == 0) trace_rec(pl.trace, 16, sgi);
+          trace_rec(pl.trace, 16, sgi, iss == 0);
           if (!(pl.ablate & 2)) {  // DEBUG timing ablation: skip the MMAs (commits still signal)
 #pragma unroll
             for (int pos = 0; pos < KPS; ++pos) {
@@ -465,10 +505,10 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
               }
             }
           }
-          if (iss == 0) trace_rec(pl.trace, 17, sgi);
+          trace_rec(pl.trace, 17, sgi, iss == 0);
           if constexpr (PAIR) { mma_commit2(&st_empty[ss]); mma_commit2(&u_empty[us]); }
           else { mma_commit(&st_empty[ss]); mma_commit(&u_empty[us]); }
-          if (iss == 0) trace_rec(pl.trace, 18, sgi);
+          trace_rec(pl.trace, 18, sgi, iss == 0);
           if (++ss == NSS) { ss = 0; sph ^= 1; }
           if (++us == NUS) { us = 0; uph ^= 1; }
         }

@@ -25,9 +25,11 @@ for name in sys.argv[1:] or ["cfg2"]:
                                 torch.cuda.current_stream().cuda_stream)
         assert rc == 0
     torch.cuda.synchronize()
+    if int(tr.count_nonzero()) == 0:
+        sys.exit("no trace records: build the library with `make -C paper_conf_icpp_zhangzxyw24_b200 TRACE=1`")
     T2 = tr.cpu().numpy().reshape(2, 32, 512).astype(np.int64)
     t0 = T2[T2 > 0].min()
-    T2 = np.where(T2 > 0, T2 - t0, -1)   # ns (globaltimer)
+    T2 = np.where(T2 > 0, T2 - t0, -1)   # cycles (clock64; CTA1 not comparable)
     t = T2[0]
     def v(k, cta=0): return T2[cta][k][T2[cta][k] >= 0]
     pl = i2cw.debug_plan(kind, N, H, W, C, K, R, S, ph, pw)
@@ -39,6 +41,9 @@ for name in sys.argv[1:] or ["cfg2"]:
         if n < 2: continue
         print(f"WG{g}: {n} ks; st_empty wait med {np.median(b[:n]-a[:n]):.0f}; transform med {np.median(c[:n]-b[:n]):.0f}; "
               f"arrive->next start med {np.median(a[1:n]-c[:n-1]):.0f}; period med {np.median(np.diff(a[:n])):.0f}")
+        d_ = v(12 + g)
+        if len(d_) >= n:
+            print(f"      math+STTM issue med {np.median(d_[:n]-b[:n]):.0f}; wait::st+arrive med {np.median(c[:n]-d_[:n]):.0f}")
         fa, fb = v(19 + g), v(23 + g)
         m = min(len(fa), len(fb))
         print(f"      in_full waits med {np.median(fb[:m]-fa[:m]):.0f} max {np.max(fb[:m]-fa[:m])} sum {np.sum(fb[:m]-fa[:m])}")
@@ -71,3 +76,16 @@ for name in sys.argv[1:] or ["cfg2"]:
         print("U producer (CTA0): kg: before u_empty wait, issue time, issuer ready (u_full done)")
         for kg in range(0, 16):
             print("   ", kg, u30[kg], u31[kg], w16[kg] if kg < len(w16) else None)
+    if os.environ.get("TIMELINE"):
+        lab = {0: "start", 4: "after-slot", 8: "arrive", 19: "in_full?", 23: "in_full!"}
+        ev = []
+        for k0, name_ in lab.items():
+            for i, tt in enumerate(v(k0)):
+                ev.append((int(tt), f"{name_}[{i}]"))
+        for i, tt in enumerate(v(16)): ev.append((int(tt), f"   ISS ready[{i}]"))
+        for i, tt in enumerate(v(18)): ev.append((int(tt), f"   ISS commit[{i}]"))
+        ev.sort()
+        lo_ = int(os.environ.get("TL_FROM", "20000")); prev = None
+        for tt, s in ev:
+            if lo_ <= tt < lo_ + 12000:
+                print(f"   {tt:8d} (+{tt - prev if prev is not None else 0:5d}) {s}"); prev = tt
