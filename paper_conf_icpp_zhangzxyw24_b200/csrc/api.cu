@@ -167,16 +167,16 @@ int make_plan(int N, int H, int W, int C, int K, int R, int S, int pad_h, int pa
     pl.WBOX = bestw;
     pl.BOXB = pl.HBOX * pl.WBOX * 16;
     pl.PLANE = (pl.BOXB + 127) / 128 * 128;
-    // Output staging: one output column i of every tile, NT/2 channels per warpgroup
-    // (one 128- or 64-byte swizzled row per tile), stored by TMA with Q stride m.
+    // Output staging: one output column i of every tile for one warpgroup's 16 channels (one
+    // 64-byte swizzled row per tile), stored by TMA with Q stride m.
     pl.OPITCH = pl.TS * pl.m;
-    pl.OSB = pl.ROWS * pl.TS * (pl.NT / nwg_for(pl.NT)) * 4;
+    pl.OSB = pl.ROWS * pl.TS * 16 * 4;
     pl.OSTRIDE = (pl.OSB + 1023) / 1024 * 1024;
     // ring depths, most preferred first: U slots hide the L2 latency of the filter
     // stream (~1-2K cycles), input stages that of the row boxes, 2 output buffers
-    // overlap the TMA store of one output column with the next.
-    static const int kDepths[][3] = {{8, 3, 2}, {8, 3, 1}, {6, 3, 2}, {6, 3, 1}, {6, 2, 1},
-                                     {4, 3, 1}, {4, 2, 1}, {3, 2, 1}, {2, 2, 1}};
+    // overlap the TMA store of one output column with the next column's math.
+    static const int kDepths[][3] = {{8, 3, 3}, {8, 3, 2}, {6, 3, 3}, {6, 3, 2}, {6, 2, 2}, {4, 3, 2}, {4, 2, 2},
+                                     {3, 2, 2}, {2, 2, 2}};
     bool fit = false;
     const int kps = kps_for(pl.alpha, pl.NT);  // k-steps per U super-slot
     for (const auto& d : kDepths) {
@@ -231,19 +231,22 @@ int encode_x_map(const Plan& pl, const float* x, CUtensorMap* map) {
   return r == CUDA_SUCCESS ? I2CW_OK : I2CW_EUNSUPPORTED;
 }
 
-// y: [N][P][Q][K] fp32; store box = NT/2 channels x (TS*m columns walked with element
-// stride m, i.e. TS positions q0 + i) x ROWS rows x 1 image, 128B/64B swizzled.
+// y: [N][P][Q][K] fp32; store box = 16 channels x (TS*m columns walked with element
+// stride m, i.e. TS positions q0 + i) x ROWS rows x 1 image, 64B swizzled.
 // Elements outside [0,K) x [0,Q) x [0,P) are clipped by the TMA unit (the in-kernel boundary).
 int encode_y_map(const Plan& pl, float* y, CUtensorMap* map) {
   PFN_encodeTiled_t enc = get_encode();
   if (!enc) return I2CW_ECUDA;
-  const int cpw = pl.NT / nwg_for(pl.NT);
   cuuint64_t dims[4] = {(cuuint64_t)pl.K, (cuuint64_t)pl.Q, (cuuint64_t)pl.P, (cuuint64_t)pl.N};
   cuuint64_t strides[3] = {(cuuint64_t)pl.K * 4, (cuuint64_t)pl.Q * pl.K * 4, (cuuint64_t)pl.P * pl.Q * pl.K * 4};
-  cuuint32_t box[4] = {(cuuint32_t)cpw, (cuuint32_t)(pl.TS * pl.m), (cuuint32_t)pl.ROWS, 1};
+  cuuint32_t box[4] = {16u, (cuuint32_t)(pl.TS * pl.m), (cuuint32_t)pl.ROWS, 1};
   cuuint32_t es[4] = {1, (cuuint32_t)pl.m, 1, 1};
+  if (pl.ablate & 128) {  // DEBUG timing ablation: contiguous (unstrided) boxes, results wrong
+    box[1] = (cuuint32_t)pl.TS;
+    es[1] = 1;
+  }
   CUresult r = enc(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, y, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                   cpw == 32 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B,
+                   CU_TENSOR_MAP_SWIZZLE_64B,
                    CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   return r == CUDA_SUCCESS ? I2CW_OK : I2CW_EUNSUPPORTED;
 }

@@ -32,9 +32,9 @@ struct Plan {
   int GP, NPASS;        // points per pass (TMEM budget), passes = alpha / GP
   int NUS;              // U pipeline stages (v1 kernel; v2 uses the template NS)
   int OPITCH;           // (unused, kept for the debug plan layout)
-  int OSB;              // bytes of one output staging buffer = ROWS*TS*(NT/2)*4 (TMA store box)
+  int OSB;              // bytes of one output staging buffer = ROWS*TS*16*4 (TMA store box, 16 channels)
   int OSTRIDE;          // OSB rounded up to 1024 (swizzled TMA boxes need 1024-byte alignment)
-  int NOB;              // output staging buffers per warpgroup (1 or 2)
+  int NOB;              // output staging buffers per warpgroup (1..4)
   int NIS;              // input (x row box) stages
   int smem_bytes;
   int pair;             // 1: CTA pairs (cluster of 2) with tcgen05.mma.cta_group::2, U split by N halves
@@ -58,10 +58,13 @@ __host__ __device__ constexpr int ns_for(int alpha, int NT) {
              : (((512 - gp_for(alpha, NT) * NT) / (gp_for(alpha, NT) * 16)) / 2) * 2;
 }
 // k-steps per super-stage (one barrier round trip + one U slot): 2 when 4 V slots fit
-__host__ __device__ constexpr int kps_for(int alpha, int NT) { return ns_for(alpha, NT) >= 4 ? 2 : 1; }
-// MMA-issuing warps: one warp issues at most ~1 UMMA per 45 cycles (measured,
-// tools/mma_bench.cu), so several warps issue, each owning whole accumulators.
-__host__ __device__ constexpr int niss_for(int GP) { return GP % 4 == 0 ? 4 : (GP % 3 == 0 ? 3 : 2); }
+#ifndef I2CW_KPS_MAX
+#define I2CW_KPS_MAX 2
+#endif
+__host__ __device__ constexpr int kps_for(int alpha, int NT) { return ns_for(alpha, NT) >= 4 ? I2CW_KPS_MAX : 1; }
+// MMA-issuing warps: each owns whole accumulators (deterministic accumulation order). Two
+// warps, each issuing warp-uniformly (elect.sync inside the asm), keep up with 32-cycle UMMAs.
+__host__ __device__ constexpr int niss_for(int GP) { return GP % 2 == 0 ? 2 : 1; }
 // Transform / epilogue warpgroups: the input transform of one k-step by one
 // warpgroup (one warp per SMSP) is latency-bound, so NT=64 (4 stages) uses 4
 // warpgroups, each owning one stage and 16 output channels in the epilogue.
@@ -195,6 +198,13 @@ template <int N>
 __device__ __forceinline__ void bulk_wait_group_read() {
   asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory");
 }
+// wait until at most n (runtime, <= 3; n < 0 waits for all) bulk groups are still reading smem
+__device__ __forceinline__ void bulk_wait_group_read_dyn(int n) {
+  if (n >= 3) bulk_wait_group_read<3>();
+  else if (n == 2) bulk_wait_group_read<2>();
+  else if (n == 1) bulk_wait_group_read<1>();
+  else bulk_wait_group_read<0>();
+}
 __device__ __forceinline__ void bulk_wait_group_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
 // generic-proxy shared-memory writes -> visible to the async proxy (TMA store reads)
 __device__ __forceinline__ void fence_proxy_async_smem() {
@@ -270,6 +280,16 @@ __device__ __forceinline__ void mbar_wait_tc(uint64_t* bar, uint32_t parity) {
   else mbar_wait(bar, parity);
 }
 
+// warpgroup register reallocation (all threads of the warpgroup execute it)
+template <int N>
+__device__ __forceinline__ void setmaxnreg_inc() {
+  asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(N));
+}
+template <int N>
+__device__ __forceinline__ void setmaxnreg_dec() {
+  asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(N));
+}
+
 // ---- tcgen05 --------------------------------------------------------------
 __device__ __forceinline__ void tmem_alloc2(uint32_t* smem_dst, uint32_t ncols) {
   asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(smem_dst)),
@@ -319,6 +339,44 @@ __device__ __forceinline__ void tc_fence_before() {
 __device__ __forceinline__ void tc_fence_after() {
   asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
 }
+// Warp-collective forms (all 32 lanes call with warp-uniform operands; one elected lane issues):
+// uniform operands stay in uniform registers instead of a per-call elect/broadcast loop.
+__device__ __forceinline__ void mma_tf32_ts_warp(uint32_t d_tmem, uint32_t a_tmem, uint64_t b_desc, uint32_t idesc,
+                                                 uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p, e;\n\t"
+      "elect.sync _|e, 0xffffffff;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::tf32 [%0], [%1], %2, %3, p;\n\t}" ::"r"(d_tmem),
+      "r"(a_tmem), "l"(b_desc), "r"(idesc), "r"(accumulate)
+      : "memory");
+}
+__device__ __forceinline__ void mma2_tf32_ts_warp(uint32_t d_tmem, uint32_t a_tmem, uint64_t b_desc, uint32_t idesc,
+                                                  uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p, e;\n\t"
+      "elect.sync _|e, 0xffffffff;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "@e tcgen05.mma.cta_group::2.kind::tf32 [%0], [%1], %2, %3, p;\n\t}" ::"r"(d_tmem),
+      "r"(a_tmem), "l"(b_desc), "r"(idesc), "r"(accumulate)
+      : "memory");
+}
+__device__ __forceinline__ void mma_commit_warp(uint64_t* bar) {
+  asm volatile(
+      "{\n\t.reg .pred e;\n\t"
+      "elect.sync _|e, 0xffffffff;\n\t"
+      "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n\t}" ::"r"(smem_u32(bar))
+      : "memory");
+}
+__device__ __forceinline__ void mma_commit2_warp(uint64_t* bar) {
+  asm volatile(
+      "{\n\t.reg .pred e;\n\t"
+      "elect.sync _|e, 0xffffffff;\n\t"
+      "@e tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;\n\t}" ::"r"(
+          smem_u32(bar)),
+      "h"((uint16_t)0x3)
+      : "memory");
+}
 // D[tmem] (+)= A[tmem] * B[smem]^T, kind::tf32, M=128, N from idesc, K=8
 __device__ __forceinline__ void mma_tf32_ts(uint32_t d_tmem, uint32_t a_tmem, uint64_t b_desc, uint32_t idesc,
                                             uint32_t accumulate) {
@@ -347,6 +405,17 @@ __device__ __forceinline__ void tmem_st_x4(uint32_t taddr, float a, float b, flo
   asm volatile("tcgen05.st.sync.aligned.32x32b.x4.b32 [%0], {%1, %2, %3, %4};" ::"r"(taddr), "r"(__float_as_uint(a)),
                "r"(__float_as_uint(b)), "r"(__float_as_uint(c)), "r"(__float_as_uint(d))
                : "memory");
+}
+// 16 consecutive columns of this thread's lane
+__device__ __forceinline__ void tmem_st_x16(uint32_t taddr, const float (&v)[16]) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, "
+      "%15, %16};" ::"r"(taddr),
+      "r"(__float_as_uint(v[0])), "r"(__float_as_uint(v[1])), "r"(__float_as_uint(v[2])), "r"(__float_as_uint(v[3])),
+      "r"(__float_as_uint(v[4])), "r"(__float_as_uint(v[5])), "r"(__float_as_uint(v[6])), "r"(__float_as_uint(v[7])),
+      "r"(__float_as_uint(v[8])), "r"(__float_as_uint(v[9])), "r"(__float_as_uint(v[10])), "r"(__float_as_uint(v[11])),
+      "r"(__float_as_uint(v[12])), "r"(__float_as_uint(v[13])), "r"(__float_as_uint(v[14])), "r"(__float_as_uint(v[15]))
+      : "memory");
 }
 __device__ __forceinline__ void tmem_wait_st() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
 __device__ __forceinline__ void tmem_ld_x8(uint32_t taddr, float* v) {

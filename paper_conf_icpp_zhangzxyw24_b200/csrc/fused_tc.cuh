@@ -35,6 +35,7 @@
 //    (TMA clips q >= Q, p >= P, k >= K: the in-kernel boundary). Passes > 0 use a
 //    TMA reduce-add into y (the accumulators hold GP of alpha points per pass).
 #pragma once
+#include <cstdlib>
 #include <utility>
 
 #include "common.cuh"
@@ -119,6 +120,7 @@ struct TcCfg {
   static constexpr int BROWS = PAIR ? NT / 2 : NT;    // B rows (output channels) held per CTA
   static constexpr int NTHREADS = tc_threads(GP, NT);
   static constexpr int PPI = GP / NISS;               // points per issuer
+
   static_assert(A % GP == 0 && GP % 2 == 0, "passes must hold whole ± pairs");
   static_assert(NS >= 2 && NS % NWG == 0, "stage ring");
   static_assert(GP * NT + NS * GP * 16 <= TMEM_COLS, "TMEM budget");
@@ -152,8 +154,12 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
   // KPS = 1, above the 384 cycles of UMMA work of a 4-point, N=64 k-step).
   constexpr int NSLOT = NS;                       // V slots in TMEM (one per warpgroup)
   static_assert(NSLOT == NWG && (NWG & (NWG - 1)) == 0, "one V slot per warpgroup, power of 2");
-  constexpr int KPS = NSLOT >= 4 ? 2 : 1;         // k-steps per super-stage
+  constexpr int KPS = kps_for(A, NT);             // k-steps per super-stage
   constexpr int NSS = NSLOT / KPS;                // super-stages
+  // epilogue: warpgroup g owns output channels [16g, 16g + 16): one 64-byte staging row per tile
+  // and output column, NOB buffers per warpgroup
+  constexpr int CPW = NT / NWG;
+  static_assert(CPW == 16, "epilogue channel split");
 
   extern __shared__ __align__(1024) uint8_t smem[];
   const uint32_t inplane = (uint32_t)pl.PLANE;  // plane stride (128-aligned)
@@ -175,26 +181,30 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(u_empty + NUS);
 
   const int warp = threadIdx.x / 32, lane32 = threadIdx.x % 32;
-  int tb, nb;
-  if constexpr (PAIR) {  // clusters of 2 along x: both CTAs share nb, take consecutive tile blocks
-    const int pr = blockIdx.x >> 1;
-    nb = pr % pl.NB;
-    tb = 2 * (pr / pl.NB) + (int)rank;
-  } else {
-    nb = blockIdx.x % pl.NB;
-    tb = blockIdx.x / pl.NB;
-  }
-  const bool cta_active = tb < pl.tile_blocks;  // odd tile-block count: the last peer only helps the MMA
-  const int seg = tb % pl.SEGS;
-  const int tbr = tb / pl.SEGS;
-  const int rb = tbr % pl.PB;
-  const int n = tbr / pl.PB;
-  const int p0 = rb * pl.ROWS;
-  // Channel-chunk rotation: CTA b walks the chunks starting at crot(b), so SMs do not all
-  // stream the same U image at the same time. Both CTAs of a pair rotate alike (their MMAs
-  // consume the same k-step). Each CTA's summation order is fixed: results stay
-  // run-to-run deterministic.
-  const int crot = (int)(((blockIdx.x >> (PAIR ? 1 : 0)) * 5u) % (unsigned)pl.NCC);
+  // Persistent schedule: a work unit is (tile block tb, output-channel block nb); CTA (pair) c
+  // takes units c, c + G, c + 2G, ... (G = number of CTAs, or of CTA pairs). Both CTAs of a
+  // pair share nb and take consecutive tile blocks. The producers run ahead across units, so
+  // the next unit's input rows and filter stream are in flight during this unit's epilogue.
+  const int NUNITS = PAIR ? ((pl.tile_blocks + 1) / 2) * pl.NB : pl.tile_blocks * pl.NB;
+  const int unit0 = PAIR ? (int)(blockIdx.x >> 1) : (int)blockIdx.x;
+  const int ustride = PAIR ? (int)(gridDim.x >> 1) : (int)gridDim.x;
+  struct Unit { int nb, tb, seg, n, p0, crot; bool active; };
+  auto unit_at = [&](int ui) {
+    Unit U;
+    U.nb = ui % pl.NB;
+    U.tb = PAIR ? 2 * (ui / pl.NB) + (int)rank : ui / pl.NB;
+    U.active = U.tb < pl.tile_blocks;  // odd tile-block count: the last peer only helps the MMA
+    U.seg = U.tb % pl.SEGS;
+    const int tbr = U.tb / pl.SEGS;
+    U.p0 = (tbr % pl.PB) * pl.ROWS;
+    U.n = tbr / pl.PB;
+    // Channel-chunk rotation: unit ui walks the chunks starting at crot, so SMs do not all
+    // stream the same U image at the same time. Both CTAs of a pair rotate alike (their MMAs
+    // consume the same k-step). The summation order is a function of the unit: results stay
+    // run-to-run deterministic.
+    U.crot = (int)(((unsigned)ui * 5u) % (unsigned)pl.NCC);
+    return U;
+  };
   const int NKS = pl.NKS;
   const int NKSP = (NKS + KPS - 1) / KPS * KPS;   // k-steps per pass padded to whole super-stages
   constexpr int PROD_WARP = NWG * 4, UPROD_WARP = NWG * 4 + 1, ISS_WARP0 = NWG * 4 + 2;
@@ -232,12 +242,12 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
     const int col0 = has_slot ? tw_l * M : 0;
     const uint32_t lane_addr = tbase + ((uint32_t)(l & ~31) << 16);
     const int TSM = pl.TS * M;  // output columns per CTA row segment
+    // Epilogue staging (warpgroup-private): buffer ob holds output column i of this warpgroup's
+    // 16 channels for every tile, one 64-byte row per tile, TMA 64B swizzle (16-byte chunk
+    // XOR (row >> 1) & 3).
     float* ostage = reinterpret_cast<float*>(o_smem + (size_t)g * pl.NOB * pl.OSTRIDE);
-    // staged row of this tile in the output box (box order: channels, tiles, rows) and its
-    // TMA swizzle: 128B rows (CPW = 32) XOR chunk with r & 7; 64B rows (CPW = 16) with (r>>1) & 3
-    constexpr int CPW = NT / NWG;
     const int orow = has_slot ? row_l * pl.TS + tw_l : 0;
-    const int oswz = CPW == 32 ? (orow & 7) : ((orow >> 1) & 3);
+    const int oswz = (orow >> 1) & 3;
     // Warpgroup g owns V slot g and computes the k-steps kg = g (mod NWG) of every pass
     // (kg = PASS * NKSP + cc * R + fh): the four warpgroups' transforms interleave on the
     // SMSPs, each k-step's full V (GP points x 8 channels, hi + lo) written by one warpgroup.
@@ -247,10 +257,15 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
       if (use > 0) mbar_wait_tc<PAIR>(&st_empty[sg % NSS], (use - 1) & 1);
     };
     int ist = 0, iph = 0;  // input ring slot / phase (incremental: no runtime division)
+    int uit = 0;           // units done by this CTA
+    for (int ui = unit0; ui < NUNITS; ui += ustride, ++uit) {
+    const Unit U = unit_at(ui);
+    const int kgb = uit * NPASS * NKSP;  // global index of this unit's first k-step
     static_for<NPASS>([&](auto PASS_) {
       constexpr int PASS = PASS_;
+      const int gpass = uit * NPASS + PASS;
       for (int cc = 0; cc < pl.NCC; ++cc) {
-        const int kb = PASS * NKSP + cc * pl.R;  // first k-step of this chunk
+        const int kb = kgb + PASS * NKSP + cc * pl.R;  // global index of the chunk's first k-step
         trace_rec(pl.trace, 19 + g, PASS * pl.NCC + cc, l == 0);
         // every warpgroup waits for every chunk (also one it has no k-step in, R < NWG) so
         // its in_empty arrival can never run ahead into the slot's next phase
@@ -260,12 +275,15 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
         for (int fh = (g - kb) & (NWG - 1); fh < pl.R; fh += NWG) {
           const int kg = kb + fh;
           trace_rec(pl.trace, 0 + g, kg / NWG, l == 0);
-          wait_slot(kg);
-          tc_fence_after();
-          trace_rec(pl.trace, 4 + g, kg / NWG, l == 0);
+          // V for this k-step computed into registers BEFORE waiting for the V slot: the slot
+          // round trip (MMA of the slot's previous k-step -> commit -> here) then covers only
+          // the split + TMEM stores, not the shared-memory loads and the B^T math.
+          float2 V[GP][4];  // point tl, channel pair cp (channels 2cp, 2cp+1 of the chunk)
           if (pl.ablate & 1) {  // DEBUG timing ablation: V = 0 without loads or math
 #pragma unroll
-            for (int c = 0; c < GP * 4; ++c) tmem_st_x4(vbase + c * 4, 0.f, 0.f, 0.f, 0.f);
+            for (int t = 0; t < GP; ++t)
+#pragma unroll
+              for (int cp = 0; cp < 4; ++cp) V[t][cp] = make_float2(0.f, 0.f);
           } else {
             const int off = (has_slot ? (row_l + fh) : 0) * pl.WBOX + col0;
 #pragma unroll
@@ -281,30 +299,37 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
               static_for<GP / 2>([&](auto Q_) {
                 constexpr int idx0 = PASS * GP + 2 * (int)Q_;  // internal index of this pair slot
                 constexpr int tl0 = 2 * (int)Q_;
-                float2 ha[2], la[2], hb[2], lb[2];
 #pragma unroll
                 for (int p = 0; p < 2; ++p) {
-                  float2 va, vb;
                   if constexpr (idx0 == 0) {  // singles: point 0 and point alpha-1
-                    va = bt_dot2<T, 0, 1, 0>(d, p);
-                    vb = bt_dot2<T, A - 1, 1, 0>(d, p);
+                    V[tl0][2 * h + p] = bt_dot2<T, 0, 1, 0>(d, p);
+                    V[tl0 + 1][2 * h + p] = bt_dot2<T, A - 1, 1, 0>(d, p);
                   } else {  // ± pair (a, a+1): E over even j, O over odd j
                     constexpr int pa = point_of(idx0, A);
                     const float2 E = bt_dot2<T, pa, 2, 0>(d, p);
                     const float2 O = bt_dot2<T, pa, 2, 1>(d, p);
-                    va = __fadd2_rn(E, O);
-                    vb = __ffma2_rn(make_float2(-1.f, -1.f), O, E);
+                    V[tl0][2 * h + p] = __fadd2_rn(E, O);
+                    V[tl0 + 1][2 * h + p] = __ffma2_rn(make_float2(-1.f, -1.f), O, E);
                   }
-                  split_tf32x2(va, ha[p], la[p]);
-                  split_tf32x2(vb, hb[p], lb[p]);
                 }
-                const uint32_t ca = vbase + tl0 * 16 + h * 4, cb = ca + 16;
-                tmem_st_x4(ca, ha[0].x, ha[0].y, ha[1].x, ha[1].y);
-                tmem_st_x4(ca + 8, la[0].x, la[0].y, la[1].x, la[1].y);
-                tmem_st_x4(cb, hb[0].x, hb[0].y, hb[1].x, hb[1].y);
-                tmem_st_x4(cb + 8, lb[0].x, lb[0].y, lb[1].x, lb[1].y);
               });
             }
+          }
+          wait_slot(kg);
+          tc_fence_after();
+          trace_rec(pl.trace, 4 + g, kg / NWG, l == 0);
+          // point tl -> 16 TMEM columns: hi of channels 0..7, then lo of channels 0..7
+#pragma unroll
+          for (int t = 0; t < GP; ++t) {
+            float v16[16];
+#pragma unroll
+            for (int cp = 0; cp < 4; ++cp) {
+              float2 hi, lo;
+              split_tf32x2(V[t][cp], hi, lo);
+              v16[2 * cp] = hi.x; v16[2 * cp + 1] = hi.y;
+              v16[8 + 2 * cp] = lo.x; v16[8 + 2 * cp + 1] = lo.y;
+            }
+            tmem_st_x16(vbase + t * 16, v16);
           }
           trace_rec(pl.trace, 12 + g, kg / NWG, l == 0);
           tmem_wait_st();
@@ -320,7 +345,7 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
       // padding k-steps of the last super-stage (NKS not a multiple of KPS): no V, but the
       // owning warpgroup still takes its turn so the super-stage's arrival count is met
       for (int kl = NKS; kl < NKSP; ++kl) {
-        const int kg = PASS * NKSP + kl;
+        const int kg = kgb + PASS * NKSP + kl;
         if ((kg & (NWG - 1)) != g) continue;
         wait_slot(kg);
         tc_fence_before();
@@ -328,79 +353,85 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
         if (lane32 == 0) mbar_arrive(&st_full[(kg / KPS) % NSS]);
       }
       // ---------- epilogue of this pass: y (+)= A^T M via shared memory + TMA ----------
-      trace_rec(pl.trace, 27, 2 * PASS, l == 0 && g == 0);
-      mbar_wait_tc<PAIR>(d_full, PASS & 1);  // completed by tcgen05.commit
+      trace_rec(pl.trace, 27, 2 * gpass, l == 0 && g == 0);
+      mbar_wait_tc<PAIR>(d_full, gpass & 1);  // completed by tcgen05.commit
       tc_fence_after();
-      trace_rec(pl.trace, 27, 2 * PASS + 1, l == 0 && g == 0);
-      // One output column i at a time over this warpgroup's CPW channels: every tile's
-      // y[q0 + i][cbase .. cbase+CPW) is one 128-byte (64-byte) row of the staging box,
-      // and the TMA store walks Q with element stride m (positions q0 + i of all tiles).
-      const int qbase = seg * TSM;
+      trace_rec(pl.trace, 27, 2 * gpass + 1, l == 0 && g == 0);
+      // Each accumulator is read from TMEM exactly once (TMEM reads run at 64 B/cycle/SM): the
+      // GP points x 16 channels of this warpgroup go to registers (the issuers may then start the
+      // next pass), the ± pair sums/differences are formed in place, and the M output columns
+      // are produced one at a time. Column i of every tile, y[q0 + i][16g .. 16g+16), is one
+      // 64-byte staging row; one TMA store per column writes the box, walking Q with element
+      // stride m (positions q0 + i). One named barrier per column: before it, thread 0 makes
+      // sure the store that last used the NEXT column's buffer has finished reading it.
+      const int qbase = U.seg * TSM;
       const int cbase = g * CPW;
       if (pl.ablate & 4) {  // DEBUG timing ablation: release the accumulators, no y
         tc_fence_before();
         __syncwarp();
         if (lane32 == 0) mbar_arrive(d_empty);
       } else {
+        float mv[GP][16];
+#pragma unroll
+        for (int t = 0; t < GP; ++t) tmem_ld_x16(lane_addr + t * NT + cbase, mv[t]);
+        tmem_wait_ld();
+        tc_fence_before();
+        __syncwarp();
+        if (lane32 == 0) mbar_arrive(d_empty);  // accumulators read: the next pass may overwrite them
+        static_for<GP / 2>([&](auto Q_) {  // pair (a, a+1): AT[i][a+1] = (-1)^i AT[i][a]
+          constexpr int idx0 = PASS * GP + 2 * (int)Q_;
+          constexpr int tl0 = 2 * (int)Q_;
+          if constexpr (idx0 != 0) {
+#pragma unroll
+            for (int e = 0; e < 16; ++e) {
+              const float sa = mv[tl0][e] + mv[tl0 + 1][e], da = mv[tl0][e] - mv[tl0 + 1][e];
+              mv[tl0][e] = sa;
+              mv[tl0 + 1][e] = da;
+            }
+          }
+        });
+        if (l == 0) bulk_wait_group_read_dyn(pl.NOB - 1);  // buffer 0: previous pass's stores
+        named_bar_sync(1 + g, 128);
         static_for<M>([&](auto I_) {
           constexpr int i = I_;
-          // staging buffer reuse: the TMA store that last read it must be done reading
           const int ob = i % pl.NOB;
-          if (l == 0) {
-            if (pl.NOB == 2) bulk_wait_group_read<1>();
-            else bulk_wait_group_read<0>();
-          }
-          named_bar_sync(1 + g, 128);
-          float4* stg = reinterpret_cast<float4*>(ostage + (size_t)ob * (pl.OSTRIDE / 4)) + (size_t)orow * (CPW / 4);
-#pragma unroll 1
-          for (int hh = 0; hh < CPW / 16; ++hh) {  // 16 channels at a time (register budget)
-            float o[16];
+          trace_rec(pl.trace, 27, 64 + 4 * (gpass * M + i), l == 0 && g == 0);
+          float4* stg = reinterpret_cast<float4*>(ostage + (size_t)ob * (pl.OSTRIDE / 4)) + (size_t)orow * 4;
 #pragma unroll
-            for (int e = 0; e < 16; ++e) o[e] = 0.f;
+          for (int j = 0; j < 4; ++j) {  // channel quads: y column i = sum over the pass's points
+            float o[4] = {0.f, 0.f, 0.f, 0.f};
             static_for<GP / 2>([&](auto Q_) {
-              constexpr int idx0 = PASS * GP + 2 * (int)Q_;  // pair slot (internal points idx0, idx0+1)
+              constexpr int idx0 = PASS * GP + 2 * (int)Q_;
               constexpr int tl0 = 2 * (int)Q_;
-              float ma[16], mb[16];
-              tmem_ld_x16(lane_addr + tl0 * NT + cbase + 16 * hh, ma);
-              tmem_ld_x16(lane_addr + (tl0 + 1) * NT + cbase + 16 * hh, mb);
-              tmem_wait_ld();
-              if constexpr (idx0 == 0) {
+              if constexpr (idx0 == 0) {  // singles: point 0 and point alpha-1
                 constexpr float c0 = T::AT(i, 0), c1 = T::AT(i, A - 1);
 #pragma unroll
-                for (int e = 0; e < 16; ++e) {
-                  if constexpr (c0 != 0.f) o[e] = fmaf(c0, ma[e], o[e]);
-                  if constexpr (c1 != 0.f) o[e] = fmaf(c1, mb[e], o[e]);
+                for (int e = 0; e < 4; ++e) {
+                  if constexpr (c0 != 0.f) o[e] = fmaf(c0, mv[tl0][4 * j + e], o[e]);
+                  if constexpr (c1 != 0.f) o[e] = fmaf(c1, mv[tl0 + 1][4 * j + e], o[e]);
                 }
-              } else {  // AT[i][a+1] = (-1)^i AT[i][a] (pair structure)
-                constexpr int pa = point_of(idx0, A);
-                constexpr float ca = T::AT(i, pa);
+              } else {
+                constexpr float ca = T::AT(i, point_of(idx0, A));
+                constexpr int src = (i % 2 == 0) ? tl0 : tl0 + 1;  // sum (even i) or difference (odd i)
 #pragma unroll
-                for (int e = 0; e < 16; ++e) {
-                  const float sv = (i % 2 == 0) ? (ma[e] + mb[e]) : (ma[e] - mb[e]);
-                  if constexpr (ca == 1.f) o[e] += sv;
-                  else if constexpr (ca != 0.f) o[e] = fmaf(ca, sv, o[e]);
+                for (int e = 0; e < 4; ++e) {
+                  if constexpr (ca == 1.f) o[e] += mv[src][4 * j + e];
+                  else if constexpr (ca != 0.f) o[e] = fmaf(ca, mv[src][4 * j + e], o[e]);
                 }
               }
             });
-            if (has_slot) {
-#pragma unroll
-              for (int j = 0; j < 4; ++j)
-                stg[(4 * hh + j) ^ oswz] = make_float4(o[4 * j], o[4 * j + 1], o[4 * j + 2], o[4 * j + 3]);
-            }
-          }
-          if constexpr (i == M - 1) {  // accumulators fully read: the issuers may start the next pass
-            tc_fence_before();
-            __syncwarp();
-            if (lane32 == 0) mbar_arrive(d_empty);
+            if (has_slot && !(pl.ablate & 64)) stg[j ^ oswz] = make_float4(o[0], o[1], o[2], o[3]);
           }
           fence_proxy_async_smem();
+          // the store that last read the next column's buffer (column i + 1 - NOB) must be done
+          if (l == 0) bulk_wait_group_read_dyn(pl.NOB - 2);
           named_bar_sync(1 + g, 128);
+          trace_rec(pl.trace, 27, 65 + 4 * (gpass * M + i), l == 0 && g == 0);
           if (l == 0) {
             const float* box = ostage + (size_t)ob * (pl.OSTRIDE / 4);
-            const int k0 = nb * NT + cbase;
-            if (cta_active) {
-              if constexpr (PASS == 0) tma_store_4d(&ymap, box, k0, qbase + i, p0, n);
-              else tma_reduce_add_4d(&ymap, box, k0, qbase + i, p0, n);
+            if (U.active && !(pl.ablate & 32)) {  // DEBUG ablation 32: no y stores
+              if constexpr (PASS == 0) tma_store_4d(&ymap, box, U.nb * NT + cbase, qbase + i, U.p0, U.n);
+              else tma_reduce_add_4d(&ymap, box, U.nb * NT + cbase, qbase + i, U.p0, U.n);
             }
             bulk_commit_group();
           }
@@ -408,31 +439,36 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
       }
       // this pass's writes must be complete before the next pass's reduce-add
       if (l == 0) bulk_wait_group_all();
-      trace_rec(pl.trace, 28, PASS, l == 0 && g == 0);
+      trace_rec(pl.trace, 28, gpass, l == 0 && g == 0);
     });
-  } else if (warp == PROD_WARP) {
+    }  // units
+  } else {
+   if (warp == PROD_WARP) {
     // ====================== input-row TMA producer ======================
     if (lane32 == 0) {
       tma_prefetch_desc(&xmap);
       tma_prefetch_desc(&ymap);
-      const int wstart = seg * pl.TS * M - pl.pad_w;
-      const int hstart = p0 - pl.pad_h;
       int ist = 0, iph = 0, first = 1;  // slot, round parity, still in the first round
+      for (int ui = unit0; ui < NUNITS; ui += ustride) {
+      const Unit U = unit_at(ui);
+      const int wstart = U.seg * pl.TS * M - pl.pad_w;
+      const int hstart = U.p0 - pl.pad_h;
       for (int pass = 0; pass < NPASS; ++pass) {
         for (int cc = 0; cc < pl.NCC; ++cc) {
           if (!first) mbar_wait(&in_empty[ist], iph ^ 1);
           uint8_t* dst = in_smem + (size_t)ist * 2 * inplane;
-          const int ca = cc + crot < pl.NCC ? cc + crot : cc + crot - pl.NCC;  // actual chunk
+          const int ca = cc + U.crot < pl.NCC ? cc + U.crot : cc + U.crot - pl.NCC;  // actual chunk
           if (pl.ablate & 16) {  // DEBUG timing ablation: no input rows (stage reused as is)
             mbar_arrive(&in_full[ist]);
           } else {
             mbar_expect_tx(&in_full[ist], 2u * (uint32_t)pl.BOXB);
-            tma_load_4d(dst, &xmap, &in_full[ist], ca * 8, wstart, hstart, n);
-            tma_load_4d(dst + inplane, &xmap, &in_full[ist], ca * 8 + 4, wstart, hstart, n);
+            tma_load_4d(dst, &xmap, &in_full[ist], ca * 8, wstart, hstart, U.n);
+            tma_load_4d(dst + inplane, &xmap, &in_full[ist], ca * 8 + 4, wstart, hstart, U.n);
           }
           if (++ist == NIS) { ist = 0; iph ^= 1; first = 0; }
         }
       }
+      }  // units
     }
     __syncwarp();
   } else if (warp == UPROD_WARP) {
@@ -440,10 +476,12 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
     if (lane32 == 0) {
       const size_t kstride = (size_t)A * 2 * NT * 8;  // floats per k-step (both layouts)
       int us = 0, uph = 0, first = 1;
+      for (int ui = unit0; ui < NUNITS; ui += ustride) {
+      const Unit U = unit_at(ui);
       for (int pass = 0; pass < NPASS; ++pass) {
         // this CTA's B rows of the pass's GP points, hi+lo, contiguous (pair: its N half)
-        const float* src0 = u + (PAIR ? u_offset_pair(NT, A, nb, NKS, 0, (int)rank, pass * GP)
-                                      : u_offset(NT, A, nb, NKS, 0, pass * GP, 0));
+        const float* src0 = u + (PAIR ? u_offset_pair(NT, A, U.nb, NKS, 0, (int)rank, pass * GP)
+                                      : u_offset(NT, A, U.nb, NKS, 0, pass * GP, 0));
         for (int kl0 = 0; kl0 < NKSP; kl0 += KPS) {
           trace_rec(pl.trace, 30, pass * NKSP + kl0);
           if (!first) mbar_wait_tc<PAIR>(&u_empty[us], uph ^ 1);  // completed by tcgen05.commit
@@ -453,36 +491,38 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
           mbar_expect_tx(&u_full[us], (uint32_t)nreal * ub);
           for (int pos = 0; pos < nreal; ++pos) {
             const int kl = kl0 + pos, cc = kl / pl.R, fh = kl - cc * pl.R;
-            const int ca = cc + crot < pl.NCC ? cc + crot : cc + crot - pl.NCC;
+            const int ca = cc + U.crot < pl.NCC ? cc + U.crot : cc + U.crot - pl.NCC;
             bulk_load(u_smem + (size_t)us * USBYTES + (size_t)pos * UBYTES, src0 + (size_t)(ca * pl.R + fh) * kstride,
                       ub, &u_full[us]);
           }
           if (++us == NUS) { us = 0; uph ^= 1; first = 0; }
         }
       }
+      }  // units
     }
     __syncwarp();
   } else {
     // ============================= MMA issuers =============================
     const int iss = warp - ISS_WARP0;  // owns points tl = iss * PPI .. iss * PPI + PPI - 1
-    if (lane32 == 0 && rank == 0) {
+    if (rank == 0) {  // the whole warp runs the loop (warp-uniform operands); one lane issues
       constexpr uint32_t idesc = idesc_tf32(PAIR ? 256 : 128, NT);
       // descriptor of U super-slot 0, k-step 0, point 0, hi; other images = + (byte offset >> 4)
       const uint64_t bdesc0 = umma_desc_kmajor_noswizzle(smem_u32(u_smem), BROWS * 16, 128);
       int ss = 0, sph = 0, us = 0, uph = 0;  // super-stage / U super-slot and their round parities
-      int sgi = 0;
-      for (int pass = 0; pass < NPASS; ++pass) {
-        if (pass > 0) {
-          mbar_wait_tc<PAIR>(d_empty, (pass - 1) & 1);
+      int sgi = 0, gpass = 0;
+      for (int ui = unit0; ui < NUNITS; ui += ustride) {
+      for (int pass = 0; pass < NPASS; ++pass, ++gpass) {
+        if (gpass > 0) {  // the epilogue has read the previous pass's accumulators
+          mbar_wait_tc<PAIR>(d_empty, (gpass - 1) & 1);
           tc_fence_after();
         }
         for (int kl0 = 0; kl0 < NKSP; kl0 += KPS, ++sgi) {
-          trace_rec(pl.trace, 29, sgi, iss == 0);
+          trace_rec(pl.trace, 29, sgi, iss == 0 && lane32 == 0);
           mbar_wait(&st_full[ss], sph);
           mbar_wait(&u_full[us], uph);
           if constexpr (PAIR) mbar_wait_cluster(&r_full[ss], sph);  // the peer's V + U half
           tc_fence_after();
-          trace_rec(pl.trace, 16, sgi, iss == 0);
+          trace_rec(pl.trace, 16, sgi, iss == 0 && lane32 == 0);
           if (!(pl.ablate & 2)) {  // DEBUG timing ablation: skip the MMAs (commits still signal)
 #pragma unroll
             for (int pos = 0; pos < KPS; ++pos) {
@@ -499,27 +539,29 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
                   const uint32_t a = va + tl * 16 + (prod == 0 ? 8 : 0);
                   const uint64_t bd = bk + (uint64_t)(((tl * 2 + (prod == 1 ? 1 : 0)) * BROWS * 32) >> 4);
                   const uint32_t acc = (kl > 0 || prod > 0) ? 1u : 0u;
-                  if constexpr (PAIR) mma2_tf32_ts(tbase + tl * NT, a, bd, idesc, acc);
-                  else mma_tf32_ts(tbase + tl * NT, a, bd, idesc, acc);
+                  if constexpr (PAIR) mma2_tf32_ts_warp(tbase + tl * NT, a, bd, idesc, acc);
+                  else mma_tf32_ts_warp(tbase + tl * NT, a, bd, idesc, acc);
                 }
               }
             }
           }
-          trace_rec(pl.trace, 17, sgi, iss == 0);
-          if constexpr (PAIR) { mma_commit2(&st_empty[ss]); mma_commit2(&u_empty[us]); }
-          else { mma_commit(&st_empty[ss]); mma_commit(&u_empty[us]); }
-          trace_rec(pl.trace, 18, sgi, iss == 0);
+          trace_rec(pl.trace, 17, sgi, iss == 0 && lane32 == 0);
+          if constexpr (PAIR) { mma_commit2_warp(&st_empty[ss]); mma_commit2_warp(&u_empty[us]); }
+          else { mma_commit_warp(&st_empty[ss]); mma_commit_warp(&u_empty[us]); }
+          trace_rec(pl.trace, 18, sgi, iss == 0 && lane32 == 0);
           if (++ss == NSS) { ss = 0; sph ^= 1; }
           if (++us == NUS) { us = 0; uph ^= 1; }
         }
-        if constexpr (PAIR) mma_commit2(d_full);
-        else mma_commit(d_full);
+        if constexpr (PAIR) mma_commit2_warp(d_full);
+        else mma_commit_warp(d_full);
       }
+      }  // units
     } else if (PAIR && lane32 == 0 && rank == 1 && iss == 0) {
       // ===== pair peer relay: forward this CTA's super-stage readiness / D drain =====
       const uint32_t lead_rfull = mapa_shared(r_full, 0), lead_dempty = mapa_shared(d_empty, 0);
-      int ss = 0, sph = 0, us = 0, uph = 0, sgi = 0;
-      for (int pass = 0; pass < NPASS; ++pass) {
+      int ss = 0, sph = 0, us = 0, uph = 0, sgi = 0, gpass = 0;
+      for (int ui = unit0; ui < NUNITS; ui += ustride) {
+      for (int pass = 0; pass < NPASS; ++pass, ++gpass) {
         for (int kl0 = 0; kl0 < NKSP; kl0 += KPS, ++sgi) {
           mbar_wait(&st_full[ss], sph);
           mbar_wait(&u_full[us], uph);
@@ -529,14 +571,15 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
           if (++ss == NSS) { ss = 0; sph ^= 1; }
           if (++us == NUS) { us = 0; uph ^= 1; }
         }
-        if (pass + 1 < NPASS) {  // this CTA's epilogue has read its D: the leader may overwrite it
-          mbar_wait(d_empty, pass & 1);
-          tc_fence_after();
-          mbar_arrive_remote(lead_dempty);
-        }
+        // this CTA's epilogue has read its D: the leader may overwrite it
+        mbar_wait(d_empty, gpass & 1);
+        tc_fence_after();
+        mbar_arrive_remote(lead_dempty);
       }
+      }  // units
     }
     __syncwarp();
+   }
   }
 
   tc_fence_before();
@@ -549,6 +592,21 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
   }
 }
 
+// Persistent grid: one CTA (pair) per SM (pair of SMs), capped by the number of work units;
+// I2CW_GRID=<n> overrides the CTA count (experiments).
+inline int persistent_ctas(int units, int per) {
+  static int nsm = 0;
+  static const int forced = [] { const char* e = getenv("I2CW_GRID"); return e ? atoi(e) : 0; }();
+  if (nsm == 0) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || nsm <= 0) nsm = 148;
+  }
+  const int cap = forced > 0 ? forced : nsm;
+  const int slots = cap / per > 0 ? cap / per : 1;
+  return (units < slots ? units : slots) * per;
+}
+
 template <int M, int RW, int NT, bool PAIR>
 static cudaError_t launch_tc_t(const CUtensorMap& xmap, const CUtensorMap& ymap, const Plan& pl, const float* u,
                                cudaStream_t stream) {
@@ -558,7 +616,7 @@ static cudaError_t launch_tc_t(const CUtensorMap& xmap, const CUtensorMap& ymap,
   if (e != cudaSuccess) return e;
   if constexpr (PAIR) {
     cudaLaunchConfig_t cfg = {};
-    cfg.gridDim = dim3(2 * ((pl.tile_blocks + 1) / 2) * pl.NB);
+    cfg.gridDim = dim3(persistent_ctas(((pl.tile_blocks + 1) / 2) * pl.NB, 2));
     cfg.blockDim = dim3(Cfg::NTHREADS);
     cfg.dynamicSmemBytes = pl.smem_bytes;
     cfg.stream = stream;
@@ -572,7 +630,7 @@ static cudaError_t launch_tc_t(const CUtensorMap& xmap, const CUtensorMap& ymap,
     e = cudaLaunchKernelEx(&cfg, kern, xmap, ymap, pl, u);
     if (e != cudaSuccess) return e;
   } else {
-    kern<<<pl.tile_blocks * pl.NB, Cfg::NTHREADS, pl.smem_bytes, stream>>>(xmap, ymap, pl, u);
+    kern<<<persistent_ctas(pl.tile_blocks * pl.NB, 1), Cfg::NTHREADS, pl.smem_bytes, stream>>>(xmap, ymap, pl, u);
   }
   return cudaGetLastError();
 }

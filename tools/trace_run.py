@@ -89,3 +89,12 @@ for name in sys.argv[1:] or ["cfg2"]:
         for tt, s in ev:
             if lo_ <= tt < lo_ + 12000:
                 print(f"   {tt:8d} (+{tt - prev if prev is not None else 0:5d}) {s}"); prev = tt
+    e27 = T2[0][27]
+    if (e27[64:] >= 0).any():
+        print("epilogue columns (WG0 thread 0): col: bulk-wait, bar1, compute+STS+bar2, to next")
+        prev = None
+        for c in range(0, 60):
+            b = 64 + 4 * c
+            if e27[b] < 0: continue
+            nxt = e27[b + 4] if e27[b + 4] >= 0 else -1
+            print(f"   {c:3d} t={e27[b]} wait {e27[b+1]-e27[b]} bar1 {e27[b+2]-e27[b+1]} body {e27[b+3]-e27[b+2]} next {nxt-e27[b+3] if nxt>=0 else None}")
