@@ -15,7 +15,7 @@ import os
 from fractions import Fraction
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libi2cw.so")
+LIB_PATH = os.environ.get("I2CW_LIB_EXPERIMENT") or os.path.join(_HERE, "libi2cw.so")  # override: timing experiments only
 _lib = None
 
 I2CW_OK, I2CW_EINVAL, I2CW_EUNSUPPORTED, I2CW_ECUDA = 0, -1, -2, -3
@@ -203,7 +203,7 @@ def transform_matrices(m, r, point_set=0):
 
 
 PLAN_FIELDS = ("P", "Q", "m", "alpha", "NT", "NB", "NCC", "NKS", "T_r", "TS", "SEGS", "ROWS", "PB", "WBOX", "HBOX",
-               "tile_blocks", "GP", "NPASS", "NUS", "smem_bytes", "pad_h", "pad_w")
+               "tile_blocks", "GP", "NPASS", "NUS", "smem_bytes", "pad_h", "pad_w", "NI")
 
 
 def debug_plan(kind, N, H, W, C, K, R, S, pad_h, pad_w):

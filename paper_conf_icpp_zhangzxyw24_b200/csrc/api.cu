@@ -8,6 +8,7 @@
 #include <cstdint>
 #include <cstring>
 #include <mutex>
+#include <tuple>
 #include <vector>
 
 #include "../../include/i2cw.h"
@@ -54,24 +55,25 @@ bool choose(int S, Choice* c) {
 
 inline int cdiv(int a, int b) { return (a + b - 1) / b; }
 
-// lane -> (row, tile) permutation. Every 8 consecutive lanes form one quarter-warp
+// lane -> (image, row, tile) permutation. Every 8 consecutive lanes form one quarter-warp
 // shared-memory wavefront for two access patterns:
-//  * input reads (LDS.128 of 16-byte columns): bank group (row*WBOX + tw*m) mod 8;
-//  * staged output writes (swizzled 128B/64B rows r = row*TS + tw): r & 7, or (r>>1) & 3.
+//  * input reads (LDS.128 of 16-byte columns): bank group (inrow*WBOX + tw*m) mod 8,
+//    inrow = img*HBOX + row (images stacked in the staged box);
+//  * staged output writes (swizzled 64B rows r = (img*ROWS + row)*TS + tw): (r >> 1) & 3 etc.
 // Greedy: fill each group with the tile adding the fewest repeated residues.
 // Returns the summed conflict degree (0 = both conflict-free).
-int assign_lanes(int ROWS, int TS, int WBOX, int m, int cpw, unsigned char* lrow, unsigned char* ltw) {
-  struct Tile { int r, t, in, out; };
+int assign_lanes(int NI, int ROWS, int HBOX, int TS, int WBOX, int m, unsigned char* lrow, unsigned short* lin,
+                 unsigned char* ltw) {
+  struct Tile { int vr, in, t, bin, bout; };
   std::vector<Tile> pool;
-  for (int r = 0; r < ROWS; ++r)
-    for (int t = 0; t < TS; ++t) {
-      const int orow = r * TS + t;
-      // 128B rows: bank group = chunk ^ (r & 7); 64B rows: (r & 1) * 4 + (chunk ^ ((r >> 1) & 3)).
-      // Either way 8 lanes with distinct r mod 8 hit 8 distinct bank groups.
-      (void)cpw;
-      pool.push_back({r, t, (r * WBOX + t * m) % 8, orow & 7});
-    }
+  for (int i = 0; i < NI; ++i)
+    for (int r = 0; r < ROWS; ++r)
+      for (int t = 0; t < TS; ++t) {
+        const int vr = i * ROWS + r, in = i * HBOX + r;
+        pool.push_back({vr, in, t, (in * WBOX + t * m) % 8, (vr * TS + t) & 7});
+      }
   std::fill(lrow, lrow + kMaxLanes, 0xFF);
+  std::fill(lin, lin + kMaxLanes, 0);
   std::fill(ltw, ltw + kMaxLanes, 0);
   int lane = 0, cost = 0;
   std::vector<char> used(pool.size(), 0);
@@ -81,14 +83,15 @@ int assign_lanes(int ROWS, int TS, int WBOX, int m, int cpw, unsigned char* lrow
       int best = -1, bestc = 1 << 30;
       for (size_t i = 0; i < pool.size(); ++i) {
         if (used[i]) continue;
-        const int c = 2 * cin[pool[i].in] + cout_[pool[i].out];
+        const int c = 2 * cin[pool[i].bin] + cout_[pool[i].bout];
         if (c < bestc) { bestc = c; best = (int)i; }
         if (c == 0) break;
       }
       used[best] = 1;
-      cin[pool[best].in]++;
-      cout_[pool[best].out]++;
-      lrow[lane] = (unsigned char)pool[best].r;
+      cin[pool[best].bin]++;
+      cout_[pool[best].bout]++;
+      lrow[lane] = (unsigned char)pool[best].vr;
+      lin[lane] = (unsigned short)pool[best].in;
       ltw[lane] = (unsigned char)pool[best].t;
       ++lane;
     }
@@ -97,6 +100,16 @@ int assign_lanes(int ROWS, int TS, int WBOX, int m, int cpw, unsigned char* lrow
     cost += (mi - 1) + (mo - 1);
   }
   return cost;
+}
+
+int num_sms() {
+  int dev = 0, nsm = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess ||
+      cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || nsm <= 0) {
+    cudaGetLastError();  // no device (host-only planning): assume a B200
+    nsm = 148;
+  }
+  return nsm;
 }
 
 }  // namespace
@@ -134,10 +147,6 @@ int make_plan(int N, int H, int W, int C, int K, int R, int S, int pad_h, int pa
   if (ts_max < 1) return I2CW_EUNSUPPORTED;
   pl.TS = std::min(pl.T_r, ts_max);
   pl.SEGS = cdiv(pl.T_r, pl.TS);
-  int rows = pl.SEGS == 1 ? std::max(1, kMaxLanes / pl.TS) : 1;
-  rows = std::min(rows, pl.P);
-  rows = std::min(rows, 256 - (R - 1));
-  if (rows < 1) return I2CW_EUNSUPPORTED;
   // CTA pairs (tcgen05.mma.cta_group::2, each CTA stages half of U): correct (all parity tests)
   // but measured 2-4% slower than single CTAs at every config, so opt-in via I2CW_PAIR=1.
   static const bool pair_ok = [] { const char* e = getenv("I2CW_PAIR"); return e && e[0] == '1'; }();
@@ -147,53 +156,84 @@ int make_plan(int N, int H, int W, int C, int K, int R, int S, int pad_h, int pa
   pl.ablate = ablate;
   const int ubytes = pl.GP * 2 * pl.NT * 32 / (pl.pair ? 2 : 1);
   const int NS = ns_for(pl.alpha, pl.NT);
-  pl.NUS = NS;
-  pl.NOB = 2;
-  pl.NIS = 4;
+  const int kps = kps_for(pl.alpha, pl.NT);  // k-steps per U super-slot
   const int wmin = pl.TS * pl.m + S - 1;
-  for (;;) {
-    // balance rows over the row blocks of an image
-    const int pb = cdiv(pl.P, rows);
-    const int rows_bal = cdiv(pl.P, pb);
-    pl.ROWS = rows_bal;
-    pl.PB = pb;
-    pl.HBOX = pl.ROWS + R - 1;
-    int best = -1, bestw = wmin;
+  // ring depths, most preferred first: U slots hide the L2 latency of the filter
+  // stream (~1-2K cycles), input stages that of the row boxes, 2 output buffers
+  // overlap the TMA store of one output column with the next column's math.
+  static const int kDepths[][3] = {{8, 3, 3}, {8, 3, 2}, {6, 3, 3}, {6, 3, 2}, {6, 2, 2}, {4, 3, 2}, {4, 2, 2},
+                                   {3, 2, 2}, {2, 2, 2}};
+  constexpr int kNumDepths = sizeof(kDepths) / sizeof(kDepths[0]);
+  // Tile blocks = NI images x ROWS output rows x TS tiles (<= 128 UMMA lanes). Candidates are
+  // ranked by (1) persistent rounds ceil(units / #SMs) -- the makespan, (2) ring depth that
+  // fits in shared memory, (3) staged input rows per unit NI * (ROWS + R - 1), (4) units.
+  // Small images pack several per block (28x28 with m = 6: 5 tiles per row; one image per
+  // block would use 70 of 128 lanes, NI = 6 x 4 rows uses 120).
+  const int nsm = num_sms();
+  struct Cand { int rounds, depth, inrows, units, NI, rows, pb; };
+  bool have = false;
+  Cand best{};
+  // I2CW_NI=<n> (tests only) forces n images per block (even n > N: a ragged last group),
+  // so small parity cases exercise multi-image blocks
+  static const int force_ni = [] { const char* e = getenv("I2CW_NI"); return e ? atoi(e) : 0; }();
+  const int ni_lo = force_ni > 0 ? std::min(force_ni, kMaxLanes / pl.TS) : 1;
+  const int ni_max = force_ni > 0 ? ni_lo : std::min(N, kMaxLanes / pl.TS);
+  for (int ni = ni_lo; ni <= ni_max; ++ni) {
+    int rmax = std::min({kMaxLanes / (ni * pl.TS), pl.P, 256 - (R - 1)});
+    if (pl.SEGS > 1) rmax = std::min(rmax, 1);
+    int last_bal = -1;
+    for (int r = rmax; r >= 1; --r) {
+      const int pb = cdiv(pl.P, r), rb = cdiv(pl.P, pb);  // balanced rows over the row blocks
+      if (rb == last_bal) continue;
+      last_bal = rb;
+      const int hbox = rb + R - 1;
+      const int plane = (ni * hbox * (wmin + 7) * 32 + 1023) / 1024 * 512;  // half stage, upper bound (WBOX <= wmin + 7)
+      const int ostride = (ni * rb * pl.TS * 64 + 1023) / 1024 * 1024;
+      int depth = -1;
+      for (int d = 0; d < kNumDepths; ++d) {
+        const int nus = std::max(kDepths[d][0] / kps, 2);
+        const int bar_bytes = 8 * (2 * kDepths[d][1] + 3 * (NS / kps) + 2 + 2 * nus) + 16;
+        const int sm = nus * kps * ubytes + kDepths[d][1] * 2 * plane + nwg_for(pl.NT) * kDepths[d][2] * ostride +
+                       bar_bytes;
+        if (sm <= kSmemBudget) { depth = d; break; }
+      }
+      if (depth < 0 || ni * hbox > 256) continue;
+      const int units = cdiv(N, ni) * pb * pl.SEGS * pl.NB;
+      const Cand c{cdiv(units, nsm), depth, ni * hbox, units, ni, rb, pb};
+      auto key = [](const Cand& x) { return std::make_tuple(x.rounds, x.depth, x.inrows, x.units, x.NI); };
+      if (!have || key(c) < key(best)) { best = c; have = true; }
+    }
+  }
+  if (!have) return I2CW_EUNSUPPORTED;
+  pl.NI = best.NI;
+  pl.ROWS = best.rows;
+  pl.PB = best.pb;
+  pl.HBOX = pl.ROWS + R - 1;
+  {
+    int bc = -1, bestw = wmin;
     for (int wb = wmin; wb <= std::min(256, wmin + 7); ++wb) {
       unsigned char lr[kMaxLanes], lt[kMaxLanes];
-      const int c = assign_lanes(pl.ROWS, pl.TS, wb, pl.m, pl.NT / nwg_for(pl.NT), lr, lt);
-      if (best < 0 || c < best) { best = c; bestw = wb; }
+      unsigned short li[kMaxLanes];
+      const int c = assign_lanes(pl.NI, pl.ROWS, pl.HBOX, pl.TS, wb, pl.m, lr, li, lt);
+      if (bc < 0 || c < bc) { bc = c; bestw = wb; }
     }
     pl.WBOX = bestw;
-    pl.BOXB = pl.HBOX * pl.WBOX * 16;
-    pl.PLANE = (pl.BOXB + 127) / 128 * 128;
-    // Output staging: one output column i of every tile for one warpgroup's 16 channels (one
-    // 64-byte swizzled row per tile), stored by TMA with Q stride m.
-    pl.OPITCH = pl.TS * pl.m;
-    pl.OSB = pl.ROWS * pl.TS * 16 * 4;
-    pl.OSTRIDE = (pl.OSB + 1023) / 1024 * 1024;
-    // ring depths, most preferred first: U slots hide the L2 latency of the filter
-    // stream (~1-2K cycles), input stages that of the row boxes, 2 output buffers
-    // overlap the TMA store of one output column with the next column's math.
-    static const int kDepths[][3] = {{8, 3, 3}, {8, 3, 2}, {6, 3, 3}, {6, 3, 2}, {6, 2, 2}, {4, 3, 2}, {4, 2, 2},
-                                     {3, 2, 2}, {2, 2, 2}};
-    bool fit = false;
-    const int kps = kps_for(pl.alpha, pl.NT);  // k-steps per U super-slot
-    for (const auto& d : kDepths) {
-      pl.NUS = std::max(d[0] / kps, 2);  // U super-slots
-      pl.NIS = d[1];
-      pl.NOB = d[2];
-      const int bar_bytes = 8 * (2 * pl.NIS + 3 * (NS / kps) + 2 + 2 * pl.NUS) + 16;
-      pl.smem_bytes = pl.NUS * kps * ubytes + pl.NIS * 2 * pl.PLANE + nwg_for(pl.NT) * pl.NOB * pl.OSTRIDE +
-                      bar_bytes;
-      if (pl.smem_bytes <= kSmemBudget) { fit = true; break; }
-    }
-    if (fit) break;
-    if (rows > 1) { rows = rows / 2; continue; }
-    return I2CW_EUNSUPPORTED;
   }
-  assign_lanes(pl.ROWS, pl.TS, pl.WBOX, pl.m, pl.NT / nwg_for(pl.NT), pl.lane_row, pl.lane_tw);
-  pl.tile_blocks = N * pl.PB * pl.SEGS;
+  pl.BOXB = pl.NI * pl.HBOX * pl.WBOX * 32;  // one 8-channel box per input stage
+  pl.PLANE = (pl.BOXB + 1023) / 1024 * 512;   // half a stage; stages stay 1024-aligned (TMA swizzle)
+  // Output staging: one output column i of every tile for one warpgroup's 16 channels (one
+  // 64-byte swizzled row per tile), stored by TMA with Q stride m.
+  pl.OPITCH = pl.TS * pl.m;
+  pl.OSB = pl.NI * pl.ROWS * pl.TS * 16 * 4;
+  pl.OSTRIDE = (pl.OSB + 1023) / 1024 * 1024;
+  pl.NUS = std::max(kDepths[best.depth][0] / kps, 2);  // U super-slots
+  pl.NIS = kDepths[best.depth][1];
+  pl.NOB = kDepths[best.depth][2];
+  const int bar_bytes = 8 * (2 * pl.NIS + 3 * (NS / kps) + 2 + 2 * pl.NUS) + 16;
+  pl.smem_bytes = pl.NUS * kps * ubytes + pl.NIS * 2 * pl.PLANE + nwg_for(pl.NT) * pl.NOB * pl.OSTRIDE + bar_bytes;
+  if (pl.smem_bytes > kSmemBudget) return I2CW_EUNSUPPORTED;
+  assign_lanes(pl.NI, pl.ROWS, pl.HBOX, pl.TS, pl.WBOX, pl.m, pl.lane_row, pl.lane_in, pl.lane_tw);
+  pl.tile_blocks = cdiv(N, pl.NI) * pl.PB * pl.SEGS;
   *out = pl;
   return I2CW_OK;
 }
@@ -217,31 +257,31 @@ PFN_encodeTiled_t get_encode() {
   return fn;
 }
 
-// x: [N][H][W][C] fp32; box = 4 channels x WBOX columns x HBOX rows x 1 image
+// x: [N][H][W][C] fp32; box = 8 channels (32 B, 32B-swizzled) x WBOX columns x HBOX rows x NI images
 int encode_x_map(const Plan& pl, const float* x, CUtensorMap* map) {
   PFN_encodeTiled_t enc = get_encode();
   if (!enc) return I2CW_ECUDA;
   cuuint64_t dims[4] = {(cuuint64_t)pl.C, (cuuint64_t)pl.W, (cuuint64_t)pl.H, (cuuint64_t)pl.N};
   cuuint64_t strides[3] = {(cuuint64_t)pl.C * 4, (cuuint64_t)pl.W * pl.C * 4, (cuuint64_t)pl.H * pl.W * pl.C * 4};
-  cuuint32_t box[4] = {4, (cuuint32_t)pl.WBOX, (cuuint32_t)pl.HBOX, 1};
+  cuuint32_t box[4] = {8, (cuuint32_t)pl.WBOX, (cuuint32_t)pl.HBOX, (cuuint32_t)pl.NI};
   cuuint32_t es[4] = {1, 1, 1, 1};
   CUresult r = enc(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, const_cast<float*>(x), dims, strides, box, es,
-                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_32B, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   return r == CUDA_SUCCESS ? I2CW_OK : I2CW_EUNSUPPORTED;
 }
 
 // y: [N][P][Q][K] fp32; store box = 16 channels x (TS*m columns walked with element
-// stride m, i.e. TS positions q0 + i) x ROWS rows x 1 image, 64B swizzled.
+// stride m, i.e. TS positions q0 + i) x ROWS rows x NI images, 64B swizzled.
 // Elements outside [0,K) x [0,Q) x [0,P) are clipped by the TMA unit (the in-kernel boundary).
 int encode_y_map(const Plan& pl, float* y, CUtensorMap* map) {
   PFN_encodeTiled_t enc = get_encode();
   if (!enc) return I2CW_ECUDA;
   cuuint64_t dims[4] = {(cuuint64_t)pl.K, (cuuint64_t)pl.Q, (cuuint64_t)pl.P, (cuuint64_t)pl.N};
   cuuint64_t strides[3] = {(cuuint64_t)pl.K * 4, (cuuint64_t)pl.Q * pl.K * 4, (cuuint64_t)pl.P * pl.Q * pl.K * 4};
-  cuuint32_t box[4] = {16u, (cuuint32_t)(pl.TS * pl.m), (cuuint32_t)pl.ROWS, 1};
+  cuuint32_t box[4] = {16u, (cuuint32_t)(pl.TS * pl.m), (cuuint32_t)pl.ROWS, (cuuint32_t)pl.NI};
   cuuint32_t es[4] = {1, (cuuint32_t)pl.m, 1, 1};
-  if (pl.ablate & 128) {  // DEBUG timing ablation: contiguous (unstrided) boxes, results wrong
+  if (I2CW_ABLATION && (pl.ablate & 128)) {  // DEBUG timing ablation: contiguous (unstrided) boxes, results wrong
     box[1] = (cuuint32_t)pl.TS;
     es[1] = 1;
   }
@@ -538,7 +578,7 @@ I2CW_API int i2cw_debug_plan(int is_deconv, int N, int H, int W, int C, int K, i
   int rc = make_plan(N, H, W, C, K, R, S, pad_h, pad_w, is_deconv, &pl);
   if (rc != I2CW_OK) return rc;
   int v[] = {pl.P, pl.Q, pl.m, pl.alpha, pl.NT, pl.NB, pl.NCC, pl.NKS, pl.T_r, pl.TS, pl.SEGS, pl.ROWS, pl.PB,
-             pl.WBOX, pl.HBOX, pl.tile_blocks, pl.GP, pl.NPASS, pl.NUS, pl.smem_bytes, pl.pad_h, pl.pad_w};
+             pl.WBOX, pl.HBOX, pl.tile_blocks, pl.GP, pl.NPASS, pl.NUS, pl.smem_bytes, pl.pad_h, pl.pad_w, pl.NI};
   for (int i = 0; i < 32; ++i) out[i] = i < (int)(sizeof(v) / sizeof(v[0])) ? v[i] : 0;
   return I2CW_OK;
 }

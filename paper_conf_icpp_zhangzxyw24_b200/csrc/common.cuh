@@ -6,6 +6,10 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#ifndef I2CW_ABLATION
+#define I2CW_ABLATION 0  // 1: timing-ablation branches compiled in (make ABLATION=1; tools only)
+#endif
+
 namespace i2cw {
 
 constexpr int kMaxLanes = 128;  // UMMA M = 128 Winograd tiles per CTA (one TMEM lane each)
@@ -25,14 +29,15 @@ struct Plan {
   int SEGS;             // segments per row = ceil(T_r / TS)
   int ROWS;             // output rows per CTA
   int PB;               // row blocks per image = ceil(P / ROWS)
+  int NI;               // images per tile block (the block's lanes are NI x ROWS x TS tiles)
   int WBOX, HBOX;       // staged input box (columns, rows = ROWS + R - 1)
-  int BOXB;             // bytes of one TMA box (one 4-channel plane) = HBOX*WBOX*16
-  int PLANE;            // shared-memory stride between planes (BOXB rounded up to 128)
-  int tile_blocks;      // N * PB * SEGS
+  int BOXB;             // bytes of one TMA input box (8 channels) = NI*HBOX*WBOX*32
+  int PLANE;            // half an input stage (BOXB rounded up to 1024, halved)
+  int tile_blocks;      // ceil(N / NI) * PB * SEGS
   int GP, NPASS;        // points per pass (TMEM budget), passes = alpha / GP
   int NUS;              // U pipeline stages (v1 kernel; v2 uses the template NS)
   int OPITCH;           // (unused, kept for the debug plan layout)
-  int OSB;              // bytes of one output staging buffer = ROWS*TS*16*4 (TMA store box, 16 channels)
+  int OSB;              // bytes of one output staging buffer = NI*ROWS*TS*16*4 (TMA store box, 16 channels)
   int OSTRIDE;          // OSB rounded up to 1024 (swizzled TMA boxes need 1024-byte alignment)
   int NOB;              // output staging buffers per warpgroup (1..4)
   int NIS;              // input (x row box) stages
@@ -41,7 +46,8 @@ struct Plan {
   int ablate;           // DEBUG timing ablation (I2CW_ABLATE, results wrong): 1 no transform math,
                         // 2 no MMAs, 4 no epilogue math/stores; 0 in production
   unsigned long long* trace;  // debug timeline of CTA 0 (nullptr = off), see i2cw_debug_trace
-  unsigned char lane_row[kMaxLanes];  // lane -> row within block (0xFF = idle lane)
+  unsigned char lane_row[kMaxLanes];  // lane -> virtual row img*ROWS + row within block (0xFF = idle lane)
+  unsigned short lane_in[kMaxLanes];  // lane -> first input row in the staged box, img*HBOX + row
   unsigned char lane_tw[kMaxLanes];   // lane -> tile within segment
 };
 
@@ -146,8 +152,30 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
 __device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
   asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
 }
+// I2CW_WAITMODE (build-time experiment switch): 0 = try_wait (HW-chosen suspend time),
+// 1 = test_wait polling (never suspends), 2 = try_wait with an explicit 32 ns suspend hint.
+#ifndef I2CW_WAITMODE
+#define I2CW_WAITMODE 0
+#endif
 __device__ __forceinline__ bool mbar_try_wait(uint64_t* bar, uint32_t parity) {
   uint32_t ok;
+#if I2CW_WAITMODE == 1
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+      "selp.u32 %0, 1, 0, p;\n\t}"
+      : "=r"(ok)
+      : "r"(smem_u32(bar)), "r"(parity)
+      : "memory");
+#elif I2CW_WAITMODE == 2
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n\t"
+      "selp.u32 %0, 1, 0, p;\n\t}"
+      : "=r"(ok)
+      : "r"(smem_u32(bar)), "r"(parity), "r"(32u)
+      : "memory");
+#else
   asm volatile(
       "{\n\t.reg .pred p;\n\t"
       "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
@@ -155,6 +183,7 @@ __device__ __forceinline__ bool mbar_try_wait(uint64_t* bar, uint32_t parity) {
       : "=r"(ok)
       : "r"(smem_u32(bar)), "r"(parity)
       : "memory");
+#endif
   return ok != 0;
 }
 // Blocking wait with a watchdog: a protocol bug traps (launch error) after ~4 s

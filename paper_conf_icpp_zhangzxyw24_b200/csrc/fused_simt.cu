@@ -26,11 +26,11 @@ __global__ void __launch_bounds__(128) fused_simt_kernel(const __grid_constant__
   const int seg = tb % pl.SEGS;
   tb /= pl.SEGS;
   const int rb = tb % pl.PB;
-  const int n = tb / pl.PB;
-  const int row_l = pl.lane_row[lane], tw_l = pl.lane_tw[lane];
-  if (row_l == 0xFF) return;
-  const int p = rb * pl.ROWS + row_l, tw = seg * pl.TS + tw_l;
-  if (p >= pl.P || tw >= pl.T_r) return;
+  const int vrow = pl.lane_row[lane], tw_l = pl.lane_tw[lane];
+  if (vrow == 0xFF) return;
+  const int n = (tb / pl.PB) * pl.NI + vrow / pl.ROWS;
+  const int p = rb * pl.ROWS + vrow % pl.ROWS, tw = seg * pl.TS + tw_l;
+  if (n >= pl.N || p >= pl.P || tw >= pl.T_r) return;
   const int q0 = tw * M;
   for (int k8 = 0; k8 < pl.NT / 8; ++k8) {
     float acc[A][8];

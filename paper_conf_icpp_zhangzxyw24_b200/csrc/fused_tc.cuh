@@ -15,7 +15,7 @@
 //    Tiles are ROWS output rows x TS tiles of one image; lane->tile is a host
 //    permutation that spreads the 16-byte shared-memory reads over banks.
 //  * a2: a TMA warp stages, per 8-channel chunk, the (ROWS+R-1) x WBOX input
-//    rows of the block as two 16-byte channel planes (OOB zero fill = padding,
+//    rows of the block as one 8-channel (32-byte, TMA-swizzled) box (OOB zero fill = padding,
 //    PAPER.md:337-338); the rows are reused across all fh (vertical overlap)
 //    and by neighbouring windows (the (r-1) horizontal overlap, §5.4).
 //    The same warp streams each k-step's U image (1D bulk copy) into a ring.
@@ -40,6 +40,10 @@
 
 #include "common.cuh"
 #include "transforms_generated.h"
+
+// Timing ablations (I2CW_ABLATE, results wrong) exist only in builds with -DI2CW_ABLATION=1
+// (make ABLATION=1); the production kernel carries no ablation branches.
+#define ABL(b) (I2CW_ABLATION && (pl.ablate & (b)))
 
 namespace i2cw {
 
@@ -162,12 +166,12 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
   static_assert(CPW == 16, "epilogue channel split");
 
   extern __shared__ __align__(1024) uint8_t smem[];
-  const uint32_t inplane = (uint32_t)pl.PLANE;  // plane stride (128-aligned)
+  const uint32_t inplane = (uint32_t)pl.PLANE;  // half an input stage (stages 1024-aligned)
   const int NUS = pl.NUS;                         // U super-slots (runtime: SMEM budget)
   constexpr uint32_t USBYTES = KPS * UBYTES;      // one U super-slot
   uint8_t* u_smem = smem;                                        // [NUS][USBYTES]        (1024-aligned)
   uint8_t* o_smem = u_smem + (size_t)NUS * USBYTES;              // [NWG][NOB][OSTRIDE]   (1024-aligned)
-  uint8_t* in_smem = o_smem + (size_t)NWG * pl.NOB * pl.OSTRIDE;  // [NIS][2 planes][PLANE]
+  uint8_t* in_smem = o_smem + (size_t)NWG * pl.NOB * pl.OSTRIDE;  // [NIS][2 * PLANE]
   uint64_t* bars = reinterpret_cast<uint64_t*>(in_smem + (size_t)NIS * 2 * inplane);
   uint64_t* in_full = bars;             // [NIS]
   uint64_t* in_empty = in_full + NIS;   // [NIS]
@@ -197,7 +201,7 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
     U.seg = U.tb % pl.SEGS;
     const int tbr = U.tb / pl.SEGS;
     U.p0 = (tbr % pl.PB) * pl.ROWS;
-    U.n = tbr / pl.PB;
+    U.n = (tbr / pl.PB) * pl.NI;
     // Channel-chunk rotation: unit ui walks the chunks starting at crot, so SMs do not all
     // stream the same U image at the same time. Both CTAs of a pair rotate alike (their MMAs
     // consume the same k-step). The summation order is a function of the unit: results stay
@@ -233,11 +237,16 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
   tc_fence_after();
   const uint32_t tbase = *tmem_slot;
 
+  // Register split (640-thread configs launch at 96 registers per thread): the transform /
+  // epilogue warpgroups take 104, the producer + issuer warpgroup keeps 56 (the CTA's pool is
+  // only what the launch allocated: 4 x 128 x 8 <= 128 x 40 released).
+  constexpr bool kRegSplit = Cfg::NTHREADS == 640;
   if (warp < NWG * 4) {
+    if constexpr (kRegSplit) setmaxnreg_inc<104>();
     // ===================== transform + epilogue warpgroups =====================
     const int g = warp / 4;           // == its V slot (NSLOT == NWG)
     const int l = threadIdx.x % 128;  // TMEM lane == tile slot
-    const int row_l = pl.lane_row[l], tw_l = pl.lane_tw[l];
+    const int row_l = pl.lane_row[l], tw_l = pl.lane_tw[l], in_l = pl.lane_in[l];
     const bool has_slot = row_l != 0xFF;
     const int col0 = has_slot ? tw_l * M : 0;
     const uint32_t lane_addr = tbase + ((uint32_t)(l & ~31) << 16);
@@ -271,7 +280,7 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
         // its in_empty arrival can never run ahead into the slot's next phase
         mbar_wait(&in_full[ist], iph);
         trace_rec(pl.trace, 23 + g, PASS * pl.NCC + cc, l == 0);
-        const float4* planes = reinterpret_cast<const float4*>(in_smem + (size_t)ist * 2 * inplane);
+        const uint8_t* stage = in_smem + (size_t)ist * 2 * inplane;  // [NI*HBOX][WBOX][8 ch], 32B-swizzled
         for (int fh = (g - kb) & (NWG - 1); fh < pl.R; fh += NWG) {
           const int kg = kb + fh;
           trace_rec(pl.trace, 0 + g, kg / NWG, l == 0);
@@ -279,20 +288,27 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
           // round trip (MMA of the slot's previous k-step -> commit -> here) then covers only
           // the split + TMEM stores, not the shared-memory loads and the B^T math.
           float2 V[GP][4];  // point tl, channel pair cp (channels 2cp, 2cp+1 of the chunk)
-          if (pl.ablate & 1) {  // DEBUG timing ablation: V = 0 without loads or math
+          if (ABL(1)) {  // DEBUG timing ablation: V = 0 without loads or math
 #pragma unroll
             for (int t = 0; t < GP; ++t)
 #pragma unroll
               for (int cp = 0; cp < 4; ++cp) V[t][cp] = make_float2(0.f, 0.f);
           } else {
-            const int off = (has_slot ? (row_l + fh) : 0) * pl.WBOX + col0;
+            // idle lanes (has_slot false: lane_in = 0, col0 = 0) read a valid window of row fh;
+            // their V only feeds accumulator rows that are never stored. Unconditional loads
+            // avoid zeroing 16 float4 per k-step.
+            // Position xs of the staged box holds 8 channels (32 bytes); the TMA 32B swizzle
+            // stores channel quad h at 16 * (h ^ bit2(xs)), so the 8 lanes of a quarter-warp
+            // (distinct xs mod 8, host lane permutation) hit 8 distinct 16-byte bank groups.
+            const int x0 = (in_l + fh) * pl.WBOX + col0;
+            const uint8_t* xrow = stage + (size_t)x0 * 32;
 #pragma unroll
-            for (int h = 0; h < 2; ++h) {  // channel quads (input planes)
-              const float4* src = planes + (size_t)h * (inplane / 16) + off;
+            for (int h = 0; h < 2; ++h) {  // channel quads
               float2 d[A][2];
 #pragma unroll
               for (int j = 0; j < A; ++j) {
-                const float4 v = has_slot ? src[j] : make_float4(0.f, 0.f, 0.f, 0.f);
+                const int sw = ((x0 + j) & 4) << 2;  // 16 * bit2(xs)
+                const float4 v = *reinterpret_cast<const float4*>(xrow + j * 32 + (h ? 16 - sw : sw));
                 d[j][0] = make_float2(v.x, v.y);
                 d[j][1] = make_float2(v.z, v.w);
               }
@@ -321,6 +337,7 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
           // point tl -> 16 TMEM columns: hi of channels 0..7, then lo of channels 0..7
 #pragma unroll
           for (int t = 0; t < GP; ++t) {
+            if (ABL(256)) break;  // DEBUG timing ablation: no TMEM stores of V
             float v16[16];
 #pragma unroll
             for (int cp = 0; cp < 4; ++cp) {
@@ -366,7 +383,7 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
       // sure the store that last used the NEXT column's buffer has finished reading it.
       const int qbase = U.seg * TSM;
       const int cbase = g * CPW;
-      if (pl.ablate & 4) {  // DEBUG timing ablation: release the accumulators, no y
+      if (ABL(4)) {  // DEBUG timing ablation: release the accumulators, no y
         tc_fence_before();
         __syncwarp();
         if (lane32 == 0) mbar_arrive(d_empty);
@@ -420,7 +437,7 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
                 }
               }
             });
-            if (has_slot && !(pl.ablate & 64)) stg[j ^ oswz] = make_float4(o[0], o[1], o[2], o[3]);
+            if (has_slot && !(ABL(64))) stg[j ^ oswz] = make_float4(o[0], o[1], o[2], o[3]);
           }
           fence_proxy_async_smem();
           // the store that last read the next column's buffer (column i + 1 - NOB) must be done
@@ -429,7 +446,7 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
           trace_rec(pl.trace, 27, 65 + 4 * (gpass * M + i), l == 0 && g == 0);
           if (l == 0) {
             const float* box = ostage + (size_t)ob * (pl.OSTRIDE / 4);
-            if (U.active && !(pl.ablate & 32)) {  // DEBUG ablation 32: no y stores
+            if (U.active && !(ABL(32))) {  // DEBUG ablation 32: no y stores
               if constexpr (PASS == 0) tma_store_4d(&ymap, box, U.nb * NT + cbase, qbase + i, U.p0, U.n);
               else tma_reduce_add_4d(&ymap, box, U.nb * NT + cbase, qbase + i, U.p0, U.n);
             }
@@ -443,6 +460,7 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
     });
     }  // units
   } else {
+   if constexpr (kRegSplit) setmaxnreg_dec<56>();
    if (warp == PROD_WARP) {
     // ====================== input-row TMA producer ======================
     if (lane32 == 0) {
@@ -458,12 +476,11 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
           if (!first) mbar_wait(&in_empty[ist], iph ^ 1);
           uint8_t* dst = in_smem + (size_t)ist * 2 * inplane;
           const int ca = cc + U.crot < pl.NCC ? cc + U.crot : cc + U.crot - pl.NCC;  // actual chunk
-          if (pl.ablate & 16) {  // DEBUG timing ablation: no input rows (stage reused as is)
+          if (ABL(16)) {  // DEBUG timing ablation: no input rows (stage reused as is)
             mbar_arrive(&in_full[ist]);
           } else {
-            mbar_expect_tx(&in_full[ist], 2u * (uint32_t)pl.BOXB);
+            mbar_expect_tx(&in_full[ist], (uint32_t)pl.BOXB);
             tma_load_4d(dst, &xmap, &in_full[ist], ca * 8, wstart, hstart, U.n);
-            tma_load_4d(dst + inplane, &xmap, &in_full[ist], ca * 8 + 4, wstart, hstart, U.n);
           }
           if (++ist == NIS) { ist = 0; iph ^= 1; first = 0; }
         }
@@ -487,7 +504,7 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
           if (!first) mbar_wait_tc<PAIR>(&u_empty[us], uph ^ 1);  // completed by tcgen05.commit
           trace_rec(pl.trace, 31, pass * NKSP + kl0);
           const int nreal = NKS - kl0 < KPS ? NKS - kl0 : KPS;
-          const uint32_t ub = (pl.ablate & 8) ? 1024u : UBYTES;  // DEBUG timing ablation: shrink
+          const uint32_t ub = (ABL(8)) ? 1024u : UBYTES;  // DEBUG timing ablation: shrink
           mbar_expect_tx(&u_full[us], (uint32_t)nreal * ub);
           for (int pos = 0; pos < nreal; ++pos) {
             const int kl = kl0 + pos, cc = kl / pl.R, fh = kl - cc * pl.R;
@@ -523,7 +540,7 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
           if constexpr (PAIR) mbar_wait_cluster(&r_full[ss], sph);  // the peer's V + U half
           tc_fence_after();
           trace_rec(pl.trace, 16, sgi, iss == 0 && lane32 == 0);
-          if (!(pl.ablate & 2)) {  // DEBUG timing ablation: skip the MMAs (commits still signal)
+          if (!(ABL(2))) {  // DEBUG timing ablation: skip the MMAs (commits still signal)
 #pragma unroll
             for (int pos = 0; pos < KPS; ++pos) {
               const int kl = kl0 + pos;

@@ -70,12 +70,12 @@ def test_planner_consistency(cfg):
     assert p["alpha"] == p["m"] + S - 1 and (p["m"], p["alpha"]) == i2cw.plan(S)[:2]
     assert p["T_r"] == -(-Q // p["m"])
     assert p["TS"] * p["SEGS"] >= p["T_r"] and p["ROWS"] * p["PB"] >= P
-    assert p["ROWS"] * p["TS"] <= 128
+    assert p["NI"] * p["ROWS"] * p["TS"] <= 128 and 1 <= p["NI"] <= N
     assert p["WBOX"] >= p["TS"] * p["m"] + S - 1 and p["WBOX"] <= 256 and p["HBOX"] == p["ROWS"] + R - 1
     assert p["GP"] * p["NPASS"] == p["alpha"] and p["GP"] * p["NT"] + 2 * 16 * p["GP"] <= 512
     assert p["NB"] * p["NT"] >= K and p["NCC"] * 8 >= C
     assert p["smem_bytes"] <= 227 * 1024
-    assert p["tile_blocks"] == N * p["PB"] * p["SEGS"]
+    assert p["tile_blocks"] == -(-N // p["NI"]) * p["PB"] * p["SEGS"]
 
 
 def test_invalid_arguments_rejected_before_cuda():

@@ -1,5 +1,6 @@
 #!/bin/bash
 # Timing ablations of the fused kernel (results are wrong under I2CW_ABLATE; timing only).
+# Needs a library built with make ABLATION=1 (the production build has no ablation branches).
 # Usage (under gpurun): bash tools/ablate.sh TAG [configs...]
 TAG=${1:-abl}; shift
 CFGS=${@:-cfg2 cfg3-r3 cfg3-r7 cfg5b-c512}
