@@ -135,7 +135,14 @@ int make_plan(int N, int H, int W, int C, int K, int R, int S, int pad_h, int pa
   if (pl.P < 1 || pl.Q < 1) return I2CW_EINVAL;
   pl.m = ch.m;
   pl.alpha = ch.alpha;
+  // Output channels per CTA (UMMA N): 64 (4 points per pass, 4 V slots of 64 columns) for
+  // K > 32, else 32. NT = 128 (2 points per pass, 8 V slots of 32 columns: a V ring twice as
+  // long in MMA time) is implemented and parity-tested but measured 10-60% slower on every
+  // K >= 128 config (twice the passes: 4 y writes per output, shallower U ring;
+  // profiles/r01f_nt128.txt), so it is opt-in: I2CW_NT=<32|64|128> overrides (experiments).
+  static const int nt_env = [] { const char* e = getenv("I2CW_NT"); return e ? atoi(e) : 0; }();
   pl.NT = K > 32 ? 64 : 32;
+  if (nt_env == 32 || nt_env == 64 || (nt_env == 128 && ch.alpha <= 12)) pl.NT = nt_env;
   pl.GP = gp_for(pl.alpha, pl.NT);
   pl.NPASS = pl.alpha / pl.GP;
   pl.NB = cdiv(K, pl.NT);
@@ -172,6 +179,7 @@ int make_plan(int N, int H, int W, int C, int K, int R, int S, int pad_h, int pa
   // Small images pack several per block (28x28 with m = 6: 5 tiles per row; one image per
   // block would use 70 of 128 lanes, NI = 6 x 4 rows uses 120).
   const int nsm = num_sms();
+  const int cpw = pl.NT / nwg_for(pl.NT);  // epilogue channels per warpgroup (staging row = cpw * 4 B)
   struct Cand { int rounds, depth, inrows, units, NI, rows, pb; };
   bool have = false;
   Cand best{};
@@ -190,7 +198,7 @@ int make_plan(int N, int H, int W, int C, int K, int R, int S, int pad_h, int pa
       last_bal = rb;
       const int hbox = rb + R - 1;
       const int plane = (ni * hbox * (wmin + 7) * 32 + 1023) / 1024 * 512;  // half stage, upper bound (WBOX <= wmin + 7)
-      const int ostride = (ni * rb * pl.TS * 64 + 1023) / 1024 * 1024;
+      const int ostride = (ni * rb * pl.TS * cpw * 4 + 1023) / 1024 * 1024;
       int depth = -1;
       for (int d = 0; d < kNumDepths; ++d) {
         const int nus = std::max(kDepths[d][0] / kps, 2);
@@ -226,7 +234,7 @@ int make_plan(int N, int H, int W, int C, int K, int R, int S, int pad_h, int pa
   // Output staging: one output column i of every tile for one warpgroup's 16 channels (one
   // 64-byte swizzled row per tile), stored by TMA with Q stride m.
   pl.OPITCH = pl.TS * pl.m;
-  pl.OSB = pl.NI * pl.ROWS * pl.TS * 16 * 4;
+  pl.OSB = pl.NI * pl.ROWS * pl.TS * cpw * 4;
   pl.OSTRIDE = (pl.OSB + 1023) / 1024 * 1024;
   pl.NUS = std::max(kDepths[best.depth][0] / kps, 2);  // U super-slots
   pl.NIS = kDepths[best.depth][1];
@@ -273,22 +281,23 @@ int encode_x_map(const Plan& pl, const float* x, CUtensorMap* map) {
   return r == CUDA_SUCCESS ? I2CW_OK : I2CW_EUNSUPPORTED;
 }
 
-// y: [N][P][Q][K] fp32; store box = 16 channels x (TS*m columns walked with element
-// stride m, i.e. TS positions q0 + i) x ROWS rows x NI images, 64B swizzled.
+// y: [N][P][Q][K] fp32; store box = NT/4 channels x (TS*m columns walked with element
+// stride m, i.e. TS positions q0 + i) x ROWS rows x NI images, 64B / 128B swizzled.
 // Elements outside [0,K) x [0,Q) x [0,P) are clipped by the TMA unit (the in-kernel boundary).
 int encode_y_map(const Plan& pl, float* y, CUtensorMap* map) {
   PFN_encodeTiled_t enc = get_encode();
   if (!enc) return I2CW_ECUDA;
   cuuint64_t dims[4] = {(cuuint64_t)pl.K, (cuuint64_t)pl.Q, (cuuint64_t)pl.P, (cuuint64_t)pl.N};
   cuuint64_t strides[3] = {(cuuint64_t)pl.K * 4, (cuuint64_t)pl.Q * pl.K * 4, (cuuint64_t)pl.P * pl.Q * pl.K * 4};
-  cuuint32_t box[4] = {16u, (cuuint32_t)(pl.TS * pl.m), (cuuint32_t)pl.ROWS, (cuuint32_t)pl.NI};
+  const int cpw = pl.NT / nwg_for(pl.NT);  // one warpgroup's channels: 64 B or 128 B rows
+  cuuint32_t box[4] = {(cuuint32_t)cpw, (cuuint32_t)(pl.TS * pl.m), (cuuint32_t)pl.ROWS, (cuuint32_t)pl.NI};
   cuuint32_t es[4] = {1, (cuuint32_t)pl.m, 1, 1};
   if (I2CW_ABLATION && (pl.ablate & 128)) {  // DEBUG timing ablation: contiguous (unstrided) boxes, results wrong
     box[1] = (cuuint32_t)pl.TS;
     es[1] = 1;
   }
   CUresult r = enc(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, y, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                   CU_TENSOR_MAP_SWIZZLE_64B,
+                   (cpw == 16 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_128B),
                    CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   return r == CUDA_SUCCESS ? I2CW_OK : I2CW_EUNSUPPORTED;
 }

@@ -51,17 +51,19 @@ struct Plan {
   unsigned char lane_tw[kMaxLanes];   // lane -> tile within segment
 };
 
-// Points per TMEM pass: GP * NT accumulator columns + 2 V stages of GP * 16
-// columns <= 512, GP even and dividing alpha.
+// Points per TMEM pass: GP * NT = 256 accumulator columns (GP even, dividing alpha; the
+// other 256 columns hold the V slots).
 __host__ __device__ constexpr int gp_for(int alpha, int NT) {
-  return NT == 64 ? 4 : (alpha % 8 == 0 ? 8 : 6);
+  return NT == 128 ? 2 : (NT == 64 ? 4 : (alpha % 8 == 0 ? 8 : 6));
 }
-// (U, V) k-step stages that fit next to the accumulators: NS * GP * 16 <= 512 - GP * NT,
-// capped at 4 and even (two transform warpgroups alternate stages).
+// V slots (one k-step of GP points, hi + lo, each) next to the accumulators:
+// NS * GP * 16 <= 512 - GP * NT. NT = 128: 8 slots of 32 columns (two per warpgroup);
+// NT = 64: 4 of 64; NT = 32: 2 of 128.
 __host__ __device__ constexpr int ns_for(int alpha, int NT) {
-  return ((512 - gp_for(alpha, NT) * NT) / (gp_for(alpha, NT) * 16)) >= 4
-             ? 4
-             : (((512 - gp_for(alpha, NT) * NT) / (gp_for(alpha, NT) * 16)) / 2) * 2;
+  return NT == 128 ? 8
+                   : (((512 - gp_for(alpha, NT) * NT) / (gp_for(alpha, NT) * 16)) >= 4
+                          ? 4
+                          : (((512 - gp_for(alpha, NT) * NT) / (gp_for(alpha, NT) * 16)) / 2) * 2);
 }
 // k-steps per super-stage (one barrier round trip + one U slot): 2 when 4 V slots fit
 #ifndef I2CW_KPS_MAX
@@ -74,7 +76,7 @@ __host__ __device__ constexpr int niss_for(int GP) { return GP % 2 == 0 ? 2 : 1;
 // Transform / epilogue warpgroups: the input transform of one k-step by one
 // warpgroup (one warp per SMSP) is latency-bound, so NT=64 (4 stages) uses 4
 // warpgroups, each owning one stage and 16 output channels in the epilogue.
-__host__ __device__ constexpr int nwg_for(int NT) { return NT == 64 ? 4 : 2; }
+__host__ __device__ constexpr int nwg_for(int NT) { return NT >= 64 ? 4 : 2; }
 __host__ __device__ constexpr int tc_threads(int GP, int NT) { return nwg_for(NT) * 128 + 64 + niss_for(GP) * 32; }
 
 // Internal Winograd point order: singles {0, alpha-1} first, then the ± pairs

@@ -156,14 +156,15 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
   // full/empty barrier pair and one U slot per super-stage, so the MMA issuers pay one
   // wait + commit per KPS k-steps (measured: ~400 cycles of barrier work per k-step with
   // KPS = 1, above the 384 cycles of UMMA work of a 4-point, N=64 k-step).
-  constexpr int NSLOT = NS;                       // V slots in TMEM (one per warpgroup)
-  static_assert(NSLOT == NWG && (NWG & (NWG - 1)) == 0, "one V slot per warpgroup, power of 2");
+  constexpr int NSLOT = NS;                       // V slots in TMEM (k-step kg uses slot kg % NSLOT)
+  static_assert(NSLOT % NWG == 0 && (NSLOT & (NSLOT - 1)) == 0 && (NWG & (NWG - 1)) == 0,
+                "V slots: a power of 2, a whole number per warpgroup");
   constexpr int KPS = kps_for(A, NT);             // k-steps per super-stage
   constexpr int NSS = NSLOT / KPS;                // super-stages
   // epilogue: warpgroup g owns output channels [16g, 16g + 16): one 64-byte staging row per tile
   // and output column, NOB buffers per warpgroup
-  constexpr int CPW = NT / NWG;
-  static_assert(CPW == 16, "epilogue channel split");
+  constexpr int CPW = NT / NWG;                   // epilogue channels per warpgroup
+  static_assert(CPW == 16 || CPW == 32, "epilogue channel split (64B / 128B staging rows)");
 
   extern __shared__ __align__(1024) uint8_t smem[];
   const uint32_t inplane = (uint32_t)pl.PLANE;  // half an input stage (stages 1024-aligned)
@@ -244,7 +245,7 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
   if (warp < NWG * 4) {
     if constexpr (kRegSplit) setmaxnreg_inc<104>();
     // ===================== transform + epilogue warpgroups =====================
-    const int g = warp / 4;           // == its V slot (NSLOT == NWG)
+    const int g = warp / 4;           // k-steps kg = g (mod NWG), V slots kg % NSLOT
     const int l = threadIdx.x % 128;  // TMEM lane == tile slot
     const int row_l = pl.lane_row[l], tw_l = pl.lane_tw[l], in_l = pl.lane_in[l];
     const bool has_slot = row_l != 0xFF;
@@ -252,15 +253,16 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
     const uint32_t lane_addr = tbase + ((uint32_t)(l & ~31) << 16);
     const int TSM = pl.TS * M;  // output columns per CTA row segment
     // Epilogue staging (warpgroup-private): buffer ob holds output column i of this warpgroup's
-    // 16 channels for every tile, one 64-byte row per tile, TMA 64B swizzle (16-byte chunk
-    // XOR (row >> 1) & 3).
+    // CPW channels for every tile, one CPW*4-byte row per tile (TMA 64B / 128B swizzle).
     float* ostage = reinterpret_cast<float*>(o_smem + (size_t)g * pl.NOB * pl.OSTRIDE);
     const int orow = has_slot ? row_l * pl.TS + tw_l : 0;
-    const int oswz = (orow >> 1) & 3;
+    // 16-byte chunk swizzle of the TMA store box rows: 64B rows (CPW 16) XOR (row >> 1) & 3,
+    // 128B rows (CPW 32) XOR row & 7
+    const int oswz = CPW == 16 ? (orow >> 1) & 3 : orow & 7;
     // Warpgroup g owns V slot g and computes the k-steps kg = g (mod NWG) of every pass
     // (kg = PASS * NKSP + cc * R + fh): the four warpgroups' transforms interleave on the
     // SMSPs, each k-step's full V (GP points x 8 channels, hi + lo) written by one warpgroup.
-    const uint32_t vbase = lane_addr + VCOL + g * GP * 16;
+    const uint32_t vbase0 = lane_addr + VCOL;
     auto wait_slot = [&](int kg) {  // this slot's previous k-step consumed (tcgen05.commit)
       const int sg = kg / KPS, use = sg / NSS;
       if (use > 0) mbar_wait_tc<PAIR>(&st_empty[sg % NSS], (use - 1) & 1);
@@ -334,6 +336,7 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
           wait_slot(kg);
           tc_fence_after();
           trace_rec(pl.trace, 4 + g, kg / NWG, l == 0);
+          const uint32_t vbase = vbase0 + (uint32_t)(kg & (NSLOT - 1)) * GP * 16;
           // point tl -> 16 TMEM columns: hi of channels 0..7, then lo of channels 0..7
 #pragma unroll
           for (int t = 0; t < GP; ++t) {
@@ -388,9 +391,11 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
         __syncwarp();
         if (lane32 == 0) mbar_arrive(d_empty);
       } else {
-        float mv[GP][16];
+        float mv[GP][CPW];
 #pragma unroll
-        for (int t = 0; t < GP; ++t) tmem_ld_x16(lane_addr + t * NT + cbase, mv[t]);
+        for (int t = 0; t < GP; ++t)
+#pragma unroll
+          for (int c16 = 0; c16 < CPW / 16; ++c16) tmem_ld_x16(lane_addr + t * NT + cbase + 16 * c16, &mv[t][16 * c16]);
         tmem_wait_ld();
         tc_fence_before();
         __syncwarp();
@@ -400,7 +405,7 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
           constexpr int tl0 = 2 * (int)Q_;
           if constexpr (idx0 != 0) {
 #pragma unroll
-            for (int e = 0; e < 16; ++e) {
+            for (int e = 0; e < CPW; ++e) {
               const float sa = mv[tl0][e] + mv[tl0 + 1][e], da = mv[tl0][e] - mv[tl0 + 1][e];
               mv[tl0][e] = sa;
               mv[tl0 + 1][e] = da;
@@ -413,9 +418,9 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
           constexpr int i = I_;
           const int ob = i % pl.NOB;
           trace_rec(pl.trace, 27, 64 + 4 * (gpass * M + i), l == 0 && g == 0);
-          float4* stg = reinterpret_cast<float4*>(ostage + (size_t)ob * (pl.OSTRIDE / 4)) + (size_t)orow * 4;
+          float4* stg = reinterpret_cast<float4*>(ostage + (size_t)ob * (pl.OSTRIDE / 4)) + (size_t)orow * (CPW / 4);
 #pragma unroll
-          for (int j = 0; j < 4; ++j) {  // channel quads: y column i = sum over the pass's points
+          for (int j = 0; j < CPW / 4; ++j) {  // channel quads: y column i = sum over the pass's points
             float o[4] = {0.f, 0.f, 0.f, 0.f};
             static_for<GP / 2>([&](auto Q_) {
               constexpr int idx0 = PASS * GP + 2 * (int)Q_;
