@@ -195,6 +195,7 @@ def main():
     import torch.distributed as dist
 
     import paper_conf_icpp_zhangzxyw24_b200 as i2cw
+    from paper_conf_icpp_zhangzxyw24_b200.shard import max_over_ranks
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -258,10 +259,7 @@ def main():
     t_total = sum(e[0].elapsed_time(e[2]) for e in evs) / 1e3        # s, K steps
     t_fused = sum(e[1].elapsed_time(e[2]) for e in evs) / 1e3
     t_ft = sum(e[0].elapsed_time(e[1]) for e in evs) / 1e3
-    tt = torch.tensor([t_total, t_fused, t_ft], dtype=torch.float64, device=dev)
-    if world > 1:
-        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-    t_total, t_fused, t_ft = tt.tolist()
+    t_total, t_fused, t_ft = max_over_ranks([t_total, t_fused, t_ft], device=dev)  # NCCL MAX (world > 1)
 
     # end-to-end through the public host-buffer call (H2D x, w + conv + D2H y every step)
     e2e = None
@@ -280,10 +278,8 @@ def main():
             i2cw.conv2d_nhwc_host(xh, wh, ph, pw, is_deconv=is_deconv, out=yh)
         eb.record(stream)
         torch.cuda.synchronize()
-        te = torch.tensor([ea.elapsed_time(eb) / 1e3], dtype=torch.float64, device=dev)
-        if world > 1:
-            dist.all_reduce(te, op=dist.ReduceOp.MAX)
-        e2e = {"value": direct_flops(cfg) * world * args.e2e_steps / te.item() / 1e12, "unit": "TFLOPS",
+        te = max_over_ranks([ea.elapsed_time(eb) / 1e3], device=dev)[0]
+        e2e = {"value": direct_flops(cfg) * world * args.e2e_steps / te / 1e12, "unit": "TFLOPS",
                "h2d_bytes_per_step": (x.numel() + w.numel()) * 4, "d2h_bytes_per_step": y.numel() * 4,
                "steps": args.e2e_steps, "api": "i2cw_conv2d_nhwc_host (pinned host buffers)"}
 
