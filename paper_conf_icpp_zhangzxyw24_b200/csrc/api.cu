@@ -174,11 +174,20 @@ int make_plan(int N, int H, int W, int C, int K, int R, int S, int pad_h, int pa
                                    {3, 2, 2}, {2, 2, 2}};
   constexpr int kNumDepths = sizeof(kDepths) / sizeof(kDepths[0]);
   // Tile blocks = NI images x ROWS output rows x TS tiles (<= 128 UMMA lanes). Candidates are
-  // ranked by (1) persistent rounds ceil(units / #SMs) -- the makespan, (2) ring depth that
+  // ranked by (1) persistent rounds ceil(units / #CTAs) -- the makespan, (2) ring depth that
   // fits in shared memory, (3) staged input rows per unit NI * (ROWS + R - 1), (4) units.
   // Small images pack several per block (28x28 with m = 6: 5 tiles per row; one image per
   // block would use 70 of 128 lanes, NI = 6 x 4 rows uses 120).
   const int nsm = num_sms();
+  // Split tail (Plan::NFULL / NITEMS, applied after the block shape is chosen): with 2 passes
+  // and no CTA pairs, the last T = units mod G units run as 2T one-pass items when 2T <= G, so
+  // they cost half a unit time (cfg2 +4%, r7 +10%). Ranking block shapes by half-unit rounds
+  // instead picked more images per block and measured slower (r2 -24%, c128 -7%), so the
+  // ranking keeps whole rounds. I2CW_SPLIT_TAIL=0 disables the split.
+  const bool split_ok = !pl.pair && pl.NPASS == 2 && [] {
+    const char* e = getenv("I2CW_SPLIT_TAIL");
+    return !(e && e[0] == '0');
+  }();
   const int cpw = pl.NT / nwg_for(pl.NT);  // epilogue channels per warpgroup (staging row = cpw * 4 B)
   struct Cand { int rounds, depth, inrows, units, NI, rows, pb; };
   bool have = false;
@@ -208,8 +217,10 @@ int make_plan(int N, int H, int W, int C, int K, int R, int S, int pad_h, int pa
         if (sm <= kSmemBudget) { depth = d; break; }
       }
       if (depth < 0 || ni * hbox > 256) continue;
-      const int units = cdiv(N, ni) * pb * pl.SEGS * pl.NB;
-      const Cand c{cdiv(units, nsm), depth, ni * hbox, units, ni, rb, pb};
+      const int blocks = cdiv(N, ni) * pb * pl.SEGS;
+      const int units = (pl.pair ? cdiv(blocks, 2) : blocks) * pl.NB;
+      const int G = pl.pair ? std::max(1, nsm / 2) : nsm;
+      const Cand c{cdiv(units, G), depth, ni * hbox, units, ni, rb, pb};
       auto key = [](const Cand& x) { return std::make_tuple(x.rounds, x.depth, x.inrows, x.units, x.NI); };
       if (!have || key(c) < key(best)) { best = c; have = true; }
     }
@@ -244,6 +255,17 @@ int make_plan(int N, int H, int W, int C, int K, int R, int S, int pad_h, int pa
   if (pl.smem_bytes > kSmemBudget) return I2CW_EUNSUPPORTED;
   assign_lanes(pl.NI, pl.ROWS, pl.HBOX, pl.TS, pl.WBOX, pl.m, pl.lane_row, pl.lane_in, pl.lane_tw);
   pl.tile_blocks = cdiv(N, pl.NI) * pl.PB * pl.SEGS;
+  {
+    const int units = (pl.pair ? cdiv(pl.tile_blocks, 2) : pl.tile_blocks) * pl.NB;
+    const int G = pl.pair ? std::max(1, nsm / 2) : nsm;
+    const int T = units % G;
+    if (split_ok && T > 0 && 2 * T <= G) {
+      pl.NFULL = units - T;
+      pl.NITEMS = pl.NFULL + 2 * T;
+    } else {
+      pl.NFULL = pl.NITEMS = units;
+    }
+  }
   *out = pl;
   return I2CW_OK;
 }
@@ -380,6 +402,15 @@ int transform_into(const Plan& pl, int is_deconv, const float* w, void* u, cudaS
 
 int run_fused(const Plan& pl, const float* x, const void* u, float* y, cudaStream_t stream) {
   CUtensorMap map, ymap;
+  if (pl.NITEMS != pl.NFULL) {
+    // split tail: both passes of a tail unit reduce-add into y, so y is zeroed from the first
+    // image the tail touches (earlier rows of that image are overwritten by whole-unit stores)
+    const int tb0 = pl.NFULL / pl.NB;
+    const size_t n0 = (size_t)(tb0 / pl.SEGS / pl.PB) * pl.NI;
+    const size_t img = (size_t)pl.P * pl.Q * pl.K;
+    if (n0 < (size_t)pl.N && cudaMemsetAsync(y + n0 * img, 0, ((size_t)pl.N - n0) * img * sizeof(float), stream) != cudaSuccess)
+      return I2CW_ECUDA;
+  }
   int rc = encode_x_map(pl, x, &map);
   if (rc != I2CW_OK) return rc;
   if ((rc = encode_y_map(pl, y, &ymap)) != I2CW_OK) return rc;
@@ -589,7 +620,8 @@ I2CW_API int i2cw_debug_plan(int is_deconv, int N, int H, int W, int C, int K, i
   int rc = make_plan(N, H, W, C, K, R, S, pad_h, pad_w, is_deconv, &pl);
   if (rc != I2CW_OK) return rc;
   int v[] = {pl.P, pl.Q, pl.m, pl.alpha, pl.NT, pl.NB, pl.NCC, pl.NKS, pl.T_r, pl.TS, pl.SEGS, pl.ROWS, pl.PB,
-             pl.WBOX, pl.HBOX, pl.tile_blocks, pl.GP, pl.NPASS, pl.NUS, pl.smem_bytes, pl.pad_h, pl.pad_w, pl.NI};
+             pl.WBOX, pl.HBOX, pl.tile_blocks, pl.GP, pl.NPASS, pl.NUS, pl.smem_bytes, pl.pad_h, pl.pad_w, pl.NI,
+             pl.NFULL, pl.NITEMS, pl.pair};
   for (int i = 0; i < 32; ++i) out[i] = i < (int)(sizeof(v) / sizeof(v[0])) ? v[i] : 0;
   return I2CW_OK;
 }

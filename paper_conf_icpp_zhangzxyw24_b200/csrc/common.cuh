@@ -34,6 +34,7 @@ struct Plan {
   int BOXB;             // bytes of one TMA input box (8 channels) = NI*HBOX*WBOX*32
   int PLANE;            // half an input stage (BOXB rounded up to 1024, halved)
   int tile_blocks;      // ceil(N / NI) * PB * SEGS
+  int NFULL, NITEMS;    // work items: [0, NFULL) whole units; then 2 per tail unit (one per pass)
   int GP, NPASS;        // points per pass (TMEM budget), passes = alpha / GP
   int NUS;              // U pipeline stages (v1 kernel; v2 uses the template NS)
   int OPITCH;           // (unused, kept for the debug plan layout)

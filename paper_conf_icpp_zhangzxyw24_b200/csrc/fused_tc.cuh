@@ -190,9 +190,20 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
   // takes units c, c + G, c + 2G, ... (G = number of CTAs, or of CTA pairs). Both CTAs of a
   // pair share nb and take consecutive tile blocks. The producers run ahead across units, so
   // the next unit's input rows and filter stream are in flight during this unit's epilogue.
-  const int NUNITS = PAIR ? ((pl.tile_blocks + 1) / 2) * pl.NB : pl.tile_blocks * pl.NB;
+  // Work items: items < NFULL are whole units (all passes); the NITEMS - NFULL items after them
+  // split the last (tail) units into one item per pass (NPASS = 2 only, y pre-zeroed by the
+  // host, both passes reduce-add: 0 + a + b is exact in either order, so results stay
+  // deterministic). A tail of T <= #CTAs/2 units then costs half a unit time instead of one.
+  const int NITEMS = pl.NITEMS;
   const int unit0 = PAIR ? (int)(blockIdx.x >> 1) : (int)blockIdx.x;
   const int ustride = PAIR ? (int)(gridDim.x >> 1) : (int)gridDim.x;
+  struct Item { int ui, pb, pe; bool split; };
+  auto item_at = [&](int it) {
+    Item I;
+    if (it < pl.NFULL) { I.ui = it; I.pb = 0; I.pe = NPASS; I.split = false; }
+    else { const int h = it - pl.NFULL; I.ui = pl.NFULL + h / 2; I.pb = h % 2; I.pe = I.pb + 1; I.split = true; }
+    return I;
+  };
   struct Unit { int nb, tb, seg, n, p0, crot; bool active; };
   auto unit_at = [&](int ui) {
     Unit U;
@@ -268,15 +279,17 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
       if (use > 0) mbar_wait_tc<PAIR>(&st_empty[sg % NSS], (use - 1) & 1);
     };
     int ist = 0, iph = 0;  // input ring slot / phase (incremental: no runtime division)
-    int uit = 0;           // units done by this CTA
-    for (int ui = unit0; ui < NUNITS; ui += ustride, ++uit) {
-    const Unit U = unit_at(ui);
-    const int kgb = uit * NPASS * NKSP;  // global index of this unit's first k-step
+    int pc = 0;            // passes done by this CTA
+    for (int it = unit0; it < NITEMS; it += ustride) {
+    const Item I = item_at(it);
+    const Unit U = unit_at(I.ui);
     static_for<NPASS>([&](auto PASS_) {
       constexpr int PASS = PASS_;
-      const int gpass = uit * NPASS + PASS;
+      if (PASS < I.pb || PASS >= I.pe) return;
+      const int gpass = pc++;
+      const int kgp = gpass * NKSP;  // global index of this pass's first k-step
       for (int cc = 0; cc < pl.NCC; ++cc) {
-        const int kb = kgb + PASS * NKSP + cc * pl.R;  // global index of the chunk's first k-step
+        const int kb = kgp + cc * pl.R;  // global index of the chunk's first k-step
         trace_rec(pl.trace, 19 + g, PASS * pl.NCC + cc, l == 0);
         // every warpgroup waits for every chunk (also one it has no k-step in, R < NWG) so
         // its in_empty arrival can never run ahead into the slot's next phase
@@ -365,7 +378,7 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
       // padding k-steps of the last super-stage (NKS not a multiple of KPS): no V, but the
       // owning warpgroup still takes its turn so the super-stage's arrival count is met
       for (int kl = NKS; kl < NKSP; ++kl) {
-        const int kg = kgb + PASS * NKSP + kl;
+        const int kg = kgp + kl;
         if ((kg & (NWG - 1)) != g) continue;
         wait_slot(kg);
         tc_fence_before();
@@ -452,7 +465,7 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
           if (l == 0) {
             const float* box = ostage + (size_t)ob * (pl.OSTRIDE / 4);
             if (U.active && !(ABL(32))) {  // DEBUG ablation 32: no y stores
-              if constexpr (PASS == 0) tma_store_4d(&ymap, box, U.nb * NT + cbase, qbase + i, U.p0, U.n);
+              if (PASS == 0 && !I.split) tma_store_4d(&ymap, box, U.nb * NT + cbase, qbase + i, U.p0, U.n);
               else tma_reduce_add_4d(&ymap, box, U.nb * NT + cbase, qbase + i, U.p0, U.n);
             }
             bulk_commit_group();
@@ -472,11 +485,12 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
       tma_prefetch_desc(&xmap);
       tma_prefetch_desc(&ymap);
       int ist = 0, iph = 0, first = 1;  // slot, round parity, still in the first round
-      for (int ui = unit0; ui < NUNITS; ui += ustride) {
-      const Unit U = unit_at(ui);
+      for (int it = unit0; it < NITEMS; it += ustride) {
+      const Item I = item_at(it);
+      const Unit U = unit_at(I.ui);
       const int wstart = U.seg * pl.TS * M - pl.pad_w;
       const int hstart = U.p0 - pl.pad_h;
-      for (int pass = 0; pass < NPASS; ++pass) {
+      for (int pass = I.pb; pass < I.pe; ++pass) {
         for (int cc = 0; cc < pl.NCC; ++cc) {
           if (!first) mbar_wait(&in_empty[ist], iph ^ 1);
           uint8_t* dst = in_smem + (size_t)ist * 2 * inplane;
@@ -498,9 +512,10 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
     if (lane32 == 0) {
       const size_t kstride = (size_t)A * 2 * NT * 8;  // floats per k-step (both layouts)
       int us = 0, uph = 0, first = 1;
-      for (int ui = unit0; ui < NUNITS; ui += ustride) {
-      const Unit U = unit_at(ui);
-      for (int pass = 0; pass < NPASS; ++pass) {
+      for (int it = unit0; it < NITEMS; it += ustride) {
+      const Item I = item_at(it);
+      const Unit U = unit_at(I.ui);
+      for (int pass = I.pb; pass < I.pe; ++pass) {
         // this CTA's B rows of the pass's GP points, hi+lo, contiguous (pair: its N half)
         const float* src0 = u + (PAIR ? u_offset_pair(NT, A, U.nb, NKS, 0, (int)rank, pass * GP)
                                       : u_offset(NT, A, U.nb, NKS, 0, pass * GP, 0));
@@ -532,8 +547,9 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
       const uint64_t bdesc0 = umma_desc_kmajor_noswizzle(smem_u32(u_smem), BROWS * 16, 128);
       int ss = 0, sph = 0, us = 0, uph = 0;  // super-stage / U super-slot and their round parities
       int sgi = 0, gpass = 0;
-      for (int ui = unit0; ui < NUNITS; ui += ustride) {
-      for (int pass = 0; pass < NPASS; ++pass, ++gpass) {
+      for (int it = unit0; it < NITEMS; it += ustride) {
+      const Item I = item_at(it);
+      for (int pass = I.pb; pass < I.pe; ++pass, ++gpass) {
         if (gpass > 0) {  // the epilogue has read the previous pass's accumulators
           mbar_wait_tc<PAIR>(d_empty, (gpass - 1) & 1);
           tc_fence_after();
@@ -582,8 +598,9 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
       // ===== pair peer relay: forward this CTA's super-stage readiness / D drain =====
       const uint32_t lead_rfull = mapa_shared(r_full, 0), lead_dempty = mapa_shared(d_empty, 0);
       int ss = 0, sph = 0, us = 0, uph = 0, sgi = 0, gpass = 0;
-      for (int ui = unit0; ui < NUNITS; ui += ustride) {
-      for (int pass = 0; pass < NPASS; ++pass, ++gpass) {
+      for (int it = unit0; it < NITEMS; it += ustride) {
+      const Item I = item_at(it);
+      for (int pass = I.pb; pass < I.pe; ++pass, ++gpass) {
         for (int kl0 = 0; kl0 < NKSP; kl0 += KPS, ++sgi) {
           mbar_wait(&st_full[ss], sph);
           mbar_wait(&u_full[us], uph);
@@ -638,7 +655,7 @@ static cudaError_t launch_tc_t(const CUtensorMap& xmap, const CUtensorMap& ymap,
   if (e != cudaSuccess) return e;
   if constexpr (PAIR) {
     cudaLaunchConfig_t cfg = {};
-    cfg.gridDim = dim3(persistent_ctas(((pl.tile_blocks + 1) / 2) * pl.NB, 2));
+    cfg.gridDim = dim3(persistent_ctas(pl.NITEMS, 2));
     cfg.blockDim = dim3(Cfg::NTHREADS);
     cfg.dynamicSmemBytes = pl.smem_bytes;
     cfg.stream = stream;
@@ -652,7 +669,7 @@ static cudaError_t launch_tc_t(const CUtensorMap& xmap, const CUtensorMap& ymap,
     e = cudaLaunchKernelEx(&cfg, kern, xmap, ymap, pl, u);
     if (e != cudaSuccess) return e;
   } else {
-    kern<<<persistent_ctas(pl.tile_blocks * pl.NB, 1), Cfg::NTHREADS, pl.smem_bytes, stream>>>(xmap, ymap, pl, u);
+    kern<<<persistent_ctas(pl.NITEMS, 1), Cfg::NTHREADS, pl.smem_bytes, stream>>>(xmap, ymap, pl, u);
   }
   return cudaGetLastError();
 }
