@@ -6,6 +6,7 @@
 
 #include <algorithm>
 #include <cstdint>
+#include <cstdio>
 #include <cstring>
 #include <mutex>
 #include <tuple>
@@ -170,9 +171,18 @@ int make_plan(int N, int H, int W, int C, int K, int R, int S, int pad_h, int pa
   // ring depths, most preferred first: U slots hide the L2 latency of the filter
   // stream (~1-2K cycles), input stages that of the row boxes, 2 output buffers
   // overlap the TMA store of one output column with the next column's math.
-  static const int kDepths[][3] = {{8, 3, 3}, {8, 3, 2}, {6, 3, 3}, {6, 3, 2}, {6, 2, 2}, {4, 3, 2}, {4, 2, 2},
-                                   {3, 2, 2}, {2, 2, 2}};
+  static int kDepths[][3] = {{8, 3, 3}, {8, 3, 2}, {6, 3, 3}, {6, 3, 2}, {6, 2, 2}, {4, 3, 2}, {4, 2, 2},
+                             {3, 2, 2}, {2, 2, 2}};
   constexpr int kNumDepths = sizeof(kDepths) / sizeof(kDepths[0]);
+  // I2CW_DEPTHS=u,i,o (experiments only): try this (U k-steps, input stages, output buffers)
+  // first
+  static const bool depth_env = [] {
+    const char* e = getenv("I2CW_DEPTHS");
+    int a, b, c;
+    if (e && sscanf(e, "%d,%d,%d", &a, &b, &c) == 3) { kDepths[0][0] = a; kDepths[0][1] = b; kDepths[0][2] = c; }
+    return e != nullptr;
+  }();
+  (void)depth_env;
   // Tile blocks = NI images x ROWS output rows x TS tiles (<= 128 UMMA lanes). Candidates are
   // ranked by (1) persistent rounds ceil(units / #CTAs) -- the makespan, (2) ring depth that
   // fits in shared memory, (3) staged input rows per unit NI * (ROWS + R - 1), (4) units.

@@ -418,10 +418,11 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
           constexpr int tl0 = 2 * (int)Q_;
           if constexpr (idx0 != 0) {
 #pragma unroll
-            for (int e = 0; e < CPW; ++e) {
-              const float sa = mv[tl0][e] + mv[tl0 + 1][e], da = mv[tl0][e] - mv[tl0 + 1][e];
-              mv[tl0][e] = sa;
-              mv[tl0 + 1][e] = da;
+            for (int e = 0; e < CPW; e += 2) {
+              const float2 a = make_float2(mv[tl0][e], mv[tl0][e + 1]), b = make_float2(mv[tl0 + 1][e], mv[tl0 + 1][e + 1]);
+              const float2 sa = __fadd2_rn(a, b), da = __ffma2_rn(make_float2(-1.f, -1.f), b, a);
+              mv[tl0][e] = sa.x; mv[tl0][e + 1] = sa.y;
+              mv[tl0 + 1][e] = da.x; mv[tl0 + 1][e + 1] = da.y;
             }
           }
         });
@@ -434,28 +435,32 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
           float4* stg = reinterpret_cast<float4*>(ostage + (size_t)ob * (pl.OSTRIDE / 4)) + (size_t)orow * (CPW / 4);
 #pragma unroll
           for (int j = 0; j < CPW / 4; ++j) {  // channel quads: y column i = sum over the pass's points
-            float o[4] = {0.f, 0.f, 0.f, 0.f};
+            // channel pairs in packed f32x2 (FFMA2 / FADD2)
+            float2 o[2] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
             static_for<GP / 2>([&](auto Q_) {
               constexpr int idx0 = PASS * GP + 2 * (int)Q_;
               constexpr int tl0 = 2 * (int)Q_;
               if constexpr (idx0 == 0) {  // singles: point 0 and point alpha-1
                 constexpr float c0 = T::AT(i, 0), c1 = T::AT(i, A - 1);
 #pragma unroll
-                for (int e = 0; e < 4; ++e) {
-                  if constexpr (c0 != 0.f) o[e] = fmaf(c0, mv[tl0][4 * j + e], o[e]);
-                  if constexpr (c1 != 0.f) o[e] = fmaf(c1, mv[tl0 + 1][4 * j + e], o[e]);
+                for (int e = 0; e < 2; ++e) {
+                  const float2 m0 = make_float2(mv[tl0][4 * j + 2 * e], mv[tl0][4 * j + 2 * e + 1]);
+                  const float2 m1 = make_float2(mv[tl0 + 1][4 * j + 2 * e], mv[tl0 + 1][4 * j + 2 * e + 1]);
+                  if constexpr (c0 != 0.f) o[e] = __ffma2_rn(make_float2(c0, c0), m0, o[e]);
+                  if constexpr (c1 != 0.f) o[e] = __ffma2_rn(make_float2(c1, c1), m1, o[e]);
                 }
               } else {
                 constexpr float ca = T::AT(i, point_of(idx0, A));
                 constexpr int src = (i % 2 == 0) ? tl0 : tl0 + 1;  // sum (even i) or difference (odd i)
 #pragma unroll
-                for (int e = 0; e < 4; ++e) {
-                  if constexpr (ca == 1.f) o[e] += mv[src][4 * j + e];
-                  else if constexpr (ca != 0.f) o[e] = fmaf(ca, mv[src][4 * j + e], o[e]);
+                for (int e = 0; e < 2; ++e) {
+                  const float2 ms = make_float2(mv[src][4 * j + 2 * e], mv[src][4 * j + 2 * e + 1]);
+                  if constexpr (ca == 1.f) o[e] = __fadd2_rn(o[e], ms);
+                  else if constexpr (ca != 0.f) o[e] = __ffma2_rn(make_float2(ca, ca), ms, o[e]);
                 }
               }
             });
-            if (has_slot && !(ABL(64))) stg[j ^ oswz] = make_float4(o[0], o[1], o[2], o[3]);
+            if (has_slot && !(ABL(64))) stg[j ^ oswz] = make_float4(o[0].x, o[0].y, o[1].x, o[1].y);
           }
           fence_proxy_async_smem();
           // the store that last read the next column's buffer (column i + 1 - NOB) must be done
