@@ -29,6 +29,7 @@ import time
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
+TF32_UBENCH_TFLOPS = 1077.0  # measured tcgen05.mma kind::tf32 128x256x8 throughput on B200
 METRIC = "direct-conv-equiv TFLOPS (fp32 NHWC, r=2..9) at 1/2/4/8 B200; % of roofline"
 
 # BASELINE.json configs; the headline (N=1 default) is configs[1], the ResNet-style 3x3 layer.
@@ -319,6 +320,10 @@ def main():
                          "work": "3xTF32 UMMA flops 6*alpha*N*P*(Q/m)*K*R*C per launch",
                          "peak_src": f"{pk_src}: bf16_tflops {pk['bf16_tflops']} x 0.5 (tf32/bf16 nominal)",
                          "hbm_frac": hbm_bytes / t_fused_launch / 1e9 / pk["hbm_gbs"],
+                         # transparency: the tf32 UMMA throughput our own microbenchmark reaches
+                         # (tools/mma_bench.cu, N = 256, 1.965 GHz) is above the nominal-ratio peak
+                         "frac_vs_ubench_tf32": achieved / TF32_UBENCH_TFLOPS,
+                         "ubench_tf32_tflops": TF32_UBENCH_TFLOPS,
                          "filter_transform_ms": t_ft / args.steps * 1e3},
             "gpu_launches": 2 * args.steps,
             "clocks": clocks,
