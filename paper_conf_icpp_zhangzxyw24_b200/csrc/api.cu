@@ -221,7 +221,7 @@ int make_plan(int N, int H, int W, int C, int K, int R, int S, int pad_h, int pa
       int depth = -1;
       for (int d = 0; d < kNumDepths; ++d) {
         const int nus = std::max(kDepths[d][0] / kps, 2);
-        const int bar_bytes = 8 * (2 * kDepths[d][1] + 3 * (NS / kps) + 2 + 2 * nus) + 16;
+        const int bar_bytes = 8 * (2 * kDepths[d][1] + NS + 2 * (NS / kps) + 2 + 2 * nus) + 16;
         const int sm = nus * kps * ubytes + kDepths[d][1] * 2 * plane + nwg_for(pl.NT) * kDepths[d][2] * ostride +
                        bar_bytes;
         if (sm <= kSmemBudget) { depth = d; break; }
@@ -260,7 +260,7 @@ int make_plan(int N, int H, int W, int C, int K, int R, int S, int pad_h, int pa
   pl.NUS = std::max(kDepths[best.depth][0] / kps, 2);  // U super-slots
   pl.NIS = kDepths[best.depth][1];
   pl.NOB = kDepths[best.depth][2];
-  const int bar_bytes = 8 * (2 * pl.NIS + 3 * (NS / kps) + 2 + 2 * pl.NUS) + 16;
+  const int bar_bytes = 8 * (2 * pl.NIS + NS + 2 * (NS / kps) + 2 + 2 * pl.NUS) + 16;
   pl.smem_bytes = pl.NUS * kps * ubytes + pl.NIS * 2 * pl.PLANE + nwg_for(pl.NT) * pl.NOB * pl.OSTRIDE + bar_bytes;
   if (pl.smem_bytes > kSmemBudget) return I2CW_EUNSUPPORTED;
   assign_lanes(pl.NI, pl.ROWS, pl.HBOX, pl.TS, pl.WBOX, pl.m, pl.lane_row, pl.lane_in, pl.lane_tw);

@@ -177,8 +177,8 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
   uint64_t* in_full = bars;             // [NIS]
   uint64_t* in_empty = in_full + NIS;   // [NIS]
   uint64_t* st_full = in_empty + NIS;   // [NSS]
-  uint64_t* st_empty = st_full + NSS;   // [NSS]
-  uint64_t* r_full = st_empty + NSS;    // [NSS]  (pair leader: the peer's super-stage relayed)
+  uint64_t* st_empty = st_full + NSS;   // [NSLOT]: one per V slot (its k-step's MMAs completed)
+  uint64_t* r_full = st_empty + NSLOT;  // [NSS]  (pair leader: the peer's super-stage relayed)
   uint64_t* d_full = r_full + NSS;      // [1]
   uint64_t* d_empty = d_full + 1;       // [1]
   uint64_t* u_full = d_empty + 1;       // [NUS]
@@ -231,9 +231,9 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
     for (int i = 0; i < NIS; ++i) { mbar_init(&in_full[i], 1); mbar_init(&in_empty[i], NWG * 4); }
     for (int i = 0; i < NSS; ++i) {
       mbar_init(&st_full[i], KPS * 4);  // the 4 warps of each of the KPS warpgroups of this super-stage
-      mbar_init(&st_empty[i], NISS);
       mbar_init(&r_full[i], 1);
     }
+    for (int i = 0; i < NSLOT; ++i) mbar_init(&st_empty[i], NISS);
     for (int i = 0; i < NUS; ++i) { mbar_init(&u_full[i], 1); mbar_init(&u_empty[i], NISS); }
     mbar_init(d_full, NISS);
     mbar_init(d_empty, NWG * 4 + (PAIR && rank == 0 ? 1 : 0));
@@ -274,9 +274,9 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
     // (kg = PASS * NKSP + cc * R + fh): the four warpgroups' transforms interleave on the
     // SMSPs, each k-step's full V (GP points x 8 channels, hi + lo) written by one warpgroup.
     const uint32_t vbase0 = lane_addr + VCOL;
-    auto wait_slot = [&](int kg) {  // this slot's previous k-step consumed (tcgen05.commit)
-      const int sg = kg / KPS, use = sg / NSS;
-      if (use > 0) mbar_wait_tc<PAIR>(&st_empty[sg % NSS], (use - 1) & 1);
+    auto wait_slot = [&](int kg) {  // this slot's previous k-step consumed (tcgen05.commit per k-step)
+      const int use = kg / NSLOT;
+      if (use > 0) mbar_wait_tc<PAIR>(&st_empty[kg & (NSLOT - 1)], (use - 1) & 1);
     };
     int ist = 0, iph = 0;  // input ring slot / phase (incremental: no runtime division)
     int pc = 0;            // passes done by this CTA
@@ -570,7 +570,14 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
 #pragma unroll
             for (int pos = 0; pos < KPS; ++pos) {
               const int kl = kl0 + pos;
-              if (kl >= NKS) break;
+              // each k-step's V slot is released by its own commit (one k-step of MMA time earlier
+              // than a per-super-stage commit for the first k-step); padding k-steps commit too
+              uint64_t* sfree = &st_empty[(sgi * KPS + pos) & (NSLOT - 1)];
+              if (kl >= NKS) {
+                if constexpr (PAIR) mma_commit2_warp(sfree);
+                else mma_commit_warp(sfree);
+                continue;
+              }
               const uint64_t bk = bdesc0 + (uint64_t)((us * USBYTES + pos * UBYTES) >> 4);
               const uint32_t va = tbase + VCOL + (ss * KPS + pos) * GP * 16;
               // product order lo*hi, hi*lo, hi*hi (small terms first), points innermost
@@ -586,11 +593,20 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
                   else mma_tf32_ts_warp(tbase + tl * NT, a, bd, idesc, acc);
                 }
               }
+              if constexpr (PAIR) mma_commit2_warp(sfree);
+              else mma_commit_warp(sfree);
+            }
+          } else {  // DEBUG ablation 2 (no MMAs): the slots are still released
+#pragma unroll
+            for (int pos = 0; pos < KPS; ++pos) {
+              uint64_t* sfree = &st_empty[(sgi * KPS + pos) & (NSLOT - 1)];
+              if constexpr (PAIR) mma_commit2_warp(sfree);
+              else mma_commit_warp(sfree);
             }
           }
           trace_rec(pl.trace, 17, sgi, iss == 0 && lane32 == 0);
-          if constexpr (PAIR) { mma_commit2_warp(&st_empty[ss]); mma_commit2_warp(&u_empty[us]); }
-          else { mma_commit_warp(&st_empty[ss]); mma_commit_warp(&u_empty[us]); }
+          if constexpr (PAIR) mma_commit2_warp(&u_empty[us]);
+          else mma_commit_warp(&u_empty[us]);
           trace_rec(pl.trace, 18, sgi, iss == 0 && lane32 == 0);
           if (++ss == NSS) { ss = 0; sph ^= 1; }
           if (++us == NUS) { us = 0; uph ^= 1; }
