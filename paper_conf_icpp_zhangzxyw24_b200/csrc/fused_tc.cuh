@@ -24,10 +24,11 @@
 //    pair trick, split 3xTF32 hi/lo and write V into TMEM
 //    with tcgen05.st (V is the UMMA A operand, "TS" mode: no SMEM read for A).
 //  * a4: NISS issuer warps, each owning GP/NISS points' accumulators, issue per
-//    k-step 3 tcgen05.mma.kind::tf32 per point (lo*hi, hi*lo, hi*hi). Several
-//    issuers are needed: one warp issues at most one UMMA per ~45 cycles while
-//    a 128x64x8 tf32 UMMA takes 32 (tools/mma_bench.cu). Each accumulator has
-//    exactly one issuer, so results are bitwise deterministic.
+//    k-step 3 tcgen05.mma.kind::tf32 per point (lo*hi, hi*lo, hi*hi). A single
+//    lane issuing in a loop manages one UMMA per ~45 cycles, a warp issuing
+//    warp-uniformly (elect.sync inside the asm) the full 32 cycles of a 128x64x8
+//    UMMA (tools/mma_bench.cu); two such warps split the points. Each accumulator
+//    has exactly one issuer, so results are bitwise deterministic.
 //  * k-step stages: NS slots, each = V (TMEM) + U (SMEM); one "full" barrier
 //    (128 transform arrivals + U tx bytes) and one "empty" barrier (NISS commits).
 //  * a5: the warpgroups tcgen05.ld the accumulators, apply A^T in registers
