@@ -123,6 +123,9 @@ I2CW_API int i2cw_deconv2d_nhwc_pretransformed(int N, int H, int W, int C, int K
  * device, runs the conv (is_deconv = 0) or deconv (is_deconv = 1) on `stream`,
  * copies y back, and synchronises `stream` before returning. Device buffers come
  * from the stream-ordered pool. Same shapes and semantics as the device calls.
+ * The batch is processed in up to 8 image chunks: host->device copies (one internal
+ * non-blocking stream) and device->host copies (another) overlap the chunks'
+ * kernels on `stream`; with pinned buffers both PCIe directions run concurrently.
  */
 I2CW_API int i2cw_conv2d_nhwc_host(int is_deconv, int N, int H, int W, int C, int K, int R, int S, int pad_h,
                           int pad_w, const float* x_host, const float* w_host, float* y_host,

@@ -554,25 +554,81 @@ int i2cw_conv2d_nhwc_host(int is_deconv, int N, int H, int W, int C, int K, int 
   int dev = 0;
   if (cudaGetDevice(&dev) != cudaSuccess) { cudaGetLastError(); return I2CW_ECUDA; }
   ensure_pool(dev);
-  const size_t xb = (size_t)N * H * W * C * 4, wb = (size_t)K * R * S * C * 4, yb = (size_t)N * pl.P * pl.Q * K * 4;
+  // Pipelined over image chunks: the host->device copy of chunk c+1 and the device->host copy
+  // of chunk c-1 run on two copy streams while chunk c computes on `stream` (PCIe is full
+  // duplex; the copies, not the kernel, bound this call). The filter is transformed once.
+  const int nchunk = std::max(1, std::min(N, 8));
+  const size_t img_x = (size_t)H * W * C, img_y = (size_t)pl.P * pl.Q * K;
+  const size_t xb = (size_t)N * img_x * 4, wb = (size_t)K * R * S * C * 4, yb = (size_t)N * img_y * 4;
+  static cudaStream_t s_in[64] = {}, s_out[64] = {};
+  static std::mutex mu;
+  {
+    std::lock_guard<std::mutex> lk(mu);
+    if (dev < 0 || dev >= 64) return I2CW_ECUDA;
+    if (!s_in[dev] && (cudaStreamCreateWithFlags(&s_in[dev], cudaStreamNonBlocking) != cudaSuccess ||
+                       cudaStreamCreateWithFlags(&s_out[dev], cudaStreamNonBlocking) != cudaSuccess)) {
+      cudaGetLastError();
+      return I2CW_ECUDA;
+    }
+  }
+  cudaStream_t si = s_in[dev], so = s_out[dev];
   float *xd = nullptr, *wd = nullptr, *yd = nullptr;
+  void* u = nullptr;
+  const size_t ub = kUTagBytes + u_data_bytes(pl);
   if (cudaMallocAsync(&xd, xb, stream) != cudaSuccess || cudaMallocAsync(&wd, wb, stream) != cudaSuccess ||
-      cudaMallocAsync(&yd, yb, stream) != cudaSuccess) {
+      cudaMallocAsync(&yd, yb, stream) != cudaSuccess || cudaMallocAsync(&u, ub, stream) != cudaSuccess) {
     cudaGetLastError();
     if (xd) cudaFreeAsync(xd, stream);
     if (wd) cudaFreeAsync(wd, stream);
+    if (yd) cudaFreeAsync(yd, stream);
     return I2CW_ECUDA;
   }
-  rc = I2CW_OK;
-  if (cudaMemcpyAsync(xd, x_host, xb, cudaMemcpyHostToDevice, stream) != cudaSuccess ||
-      cudaMemcpyAsync(wd, w_host, wb, cudaMemcpyHostToDevice, stream) != cudaSuccess)
+  std::vector<cudaEvent_t> ev(2 * nchunk + 1, nullptr);
+  for (auto& e : ev)
+    if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) rc = I2CW_ECUDA;
+  // the copy streams start after the allocations (and all earlier work) on `stream`
+  if (rc == I2CW_OK && (cudaEventRecord(ev[2 * nchunk], stream) != cudaSuccess ||
+                        cudaStreamWaitEvent(si, ev[2 * nchunk], 0) != cudaSuccess ||
+                        cudaStreamWaitEvent(so, ev[2 * nchunk], 0) != cudaSuccess))
     rc = I2CW_ECUDA;
-  if (rc == I2CW_OK) rc = conv_common(is_deconv, N, H, W, C, K, R, S, pad_h, pad_w, xd, wd, yd, stream, false);
-  if (rc == I2CW_OK && cudaMemcpyAsync(y_host, yd, yb, cudaMemcpyDeviceToHost, stream) != cudaSuccess) rc = I2CW_ECUDA;
+  if (rc == I2CW_OK && cudaMemcpyAsync(wd, w_host, wb, cudaMemcpyHostToDevice, stream) != cudaSuccess) rc = I2CW_ECUDA;
+  if (rc == I2CW_OK) rc = transform_into(pl, is_deconv, wd, u, stream);
+  int n0 = 0;
+  for (int c = 0; c < nchunk && rc == I2CW_OK; ++c) {
+    const int nc = N / nchunk + (c < N % nchunk ? 1 : 0);
+    Plan pc;
+    if ((rc = make_plan(nc, H, W, C, K, R, S, pad_h, pad_w, is_deconv, &pc)) != I2CW_OK) break;
+    float* xdc = xd + (size_t)n0 * img_x;
+    float* ydc = yd + (size_t)n0 * img_y;
+    if (cudaMemcpyAsync(xdc, x_host + (size_t)n0 * img_x, (size_t)nc * img_x * 4, cudaMemcpyHostToDevice, si) !=
+            cudaSuccess ||
+        cudaEventRecord(ev[2 * c], si) != cudaSuccess || cudaStreamWaitEvent(stream, ev[2 * c], 0) != cudaSuccess) {
+      rc = I2CW_ECUDA;
+      break;
+    }
+    if ((rc = run_fused(pc, xdc, u, ydc, stream)) != I2CW_OK) break;
+    if (cudaEventRecord(ev[2 * c + 1], stream) != cudaSuccess || cudaStreamWaitEvent(so, ev[2 * c + 1], 0) != cudaSuccess ||
+        cudaMemcpyAsync(y_host + (size_t)n0 * img_y, ydc, (size_t)nc * img_y * 4, cudaMemcpyDeviceToHost, so) !=
+            cudaSuccess) {
+      rc = I2CW_ECUDA;
+      break;
+    }
+    n0 += nc;
+  }
+  // the buffers are freed on `stream` after the last device->host copy
+  cudaEvent_t done = nullptr;
+  if (cudaEventCreateWithFlags(&done, cudaEventDisableTiming) == cudaSuccess) {
+    cudaEventRecord(done, so);
+    cudaStreamWaitEvent(stream, done, 0);
+  }
   cudaFreeAsync(xd, stream);
   cudaFreeAsync(wd, stream);
   cudaFreeAsync(yd, stream);
+  cudaFreeAsync(u, stream);
   if (cudaStreamSynchronize(stream) != cudaSuccess) rc = I2CW_ECUDA;
+  for (auto& e : ev)
+    if (e) cudaEventDestroy(e);
+  if (done) cudaEventDestroy(done);
   if (rc != I2CW_OK) cudaGetLastError();
   return rc;
 }
