@@ -18,7 +18,8 @@
 
 namespace i2cw {
 cudaError_t launch_filter_transform(const float* w, float* u, int C, int K, int R, int S, int is_deconv, int alpha,
-                                    int NT, int NB, int NCC, int halves, const double* G, cudaStream_t stream);
+                                    int NT, int NB, int NCC, int halves, const double* G, const UTag& tag,
+                                    UTag* tag_dst, cudaStream_t stream);
 cudaError_t launch_fused_tc(const CUtensorMap& xmap, const CUtensorMap& ymap, const Plan& pl, const float* u,
                             cudaStream_t stream);
 cudaError_t launch_fused_simt(const Plan& pl, const float* x, const float* u, float* y, cudaStream_t stream);
@@ -116,7 +117,7 @@ int num_sms() {
 }  // namespace
 
 // Build the launch plan. Returns I2CW_OK or an error code.
-int make_plan(int N, int H, int W, int C, int K, int R, int S, int pad_h, int pad_w, int is_deconv, Plan* out) {
+int make_plan_uncached(int N, int H, int W, int C, int K, int R, int S, int pad_h, int pad_w, int is_deconv, Plan* out) {
   Plan pl;
   std::memset(&pl, 0, sizeof(pl));
   if (N <= 0 || H <= 0 || W <= 0 || C <= 0 || K <= 0 || R <= 0 || S <= 0 || pad_h < 0 || pad_w < 0) return I2CW_EINVAL;
@@ -280,6 +281,30 @@ int make_plan(int N, int H, int W, int C, int K, int R, int S, int pad_h, int pa
   return I2CW_OK;
 }
 
+// Plans are pure functions of the call's dimensions (and the device's SM count): memoised,
+// so repeated calls skip the block-shape search and the lane permutation.
+int make_plan(int N, int H, int W, int C, int K, int R, int S, int pad_h, int pad_w, int is_deconv, Plan* out) {
+  struct Key { int v[11]; };
+  static std::mutex mu;
+  static std::vector<std::pair<Key, Plan>> memo;
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) { cudaGetLastError(); dev = -1; }
+  const Key k{{N, H, W, C, K, R, S, pad_h, pad_w, is_deconv, dev}};
+  {
+    std::lock_guard<std::mutex> lk(mu);
+    for (auto& e : memo)
+      if (std::memcmp(e.first.v, k.v, sizeof(k.v)) == 0) { *out = e.second; return I2CW_OK; }
+  }
+  Plan pl;
+  const int rc = make_plan_uncached(N, H, W, C, K, R, S, pad_h, pad_w, is_deconv, &pl);
+  if (rc != I2CW_OK) return rc;
+  std::lock_guard<std::mutex> lk(mu);
+  if (memo.size() >= 256) memo.erase(memo.begin());
+  memo.push_back({k, pl});
+  *out = pl;
+  return I2CW_OK;
+}
+
 namespace {
 
 typedef CUresult (*PFN_encodeTiled_t)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
@@ -390,22 +415,33 @@ void g_internal(const Plan& pl, int point_set, std::vector<double>* G) {
 
 size_t u_data_bytes(const Plan& pl) { return (size_t)pl.NB * pl.NKS * pl.alpha * 2 * pl.NT * 8 * 4; }
 
+// exact G tables are generated once per (m, S, point set) and kept (host memo)
+const std::vector<double>& g_cached(const Plan& pl, int point_set) {
+  static std::mutex mu;
+  static std::vector<std::pair<int, std::vector<double>>> memo;
+  const int key = (pl.m * 16 + pl.S) * 2 + point_set;
+  std::lock_guard<std::mutex> lk(mu);
+  for (auto& e : memo)
+    if (e.first == key) return e.second;
+  memo.push_back({key, {}});
+  g_internal(pl, point_set, &memo.back().second);
+  return memo.back().second;
+}
+
 int transform_into(const Plan& pl, int is_deconv, const float* w, void* u, cudaStream_t stream) {
   Choice ch;
   choose(pl.S, &ch);
-  std::vector<double> G;
-  g_internal(pl, ch.point_set, &G);
+  const std::vector<double>& G = g_cached(pl, ch.point_set);
   UTag tag;
   std::memset(&tag, 0, sizeof(tag));
   tag.magic = kUMagic; tag.alpha = pl.alpha; tag.m = pl.m; tag.is_deconv = is_deconv;
   tag.C = pl.C; tag.K = pl.K; tag.R = pl.R; tag.S = pl.S; tag.NT = pl.NT; tag.NB = pl.NB; tag.NCC = pl.NCC;
   tag.halves = pl.pair ? 2 : 1;
   static_assert(sizeof(UTag) <= kUTagBytes, "tag");
-  if (cudaMemcpyAsync(u, &tag, sizeof(tag), cudaMemcpyHostToDevice, stream) != cudaSuccess) return I2CW_ECUDA;
   registry_put(u, tag);
   float* ud = reinterpret_cast<float*>(static_cast<uint8_t*>(u) + kUTagBytes);
   if (launch_filter_transform(w, ud, pl.C, pl.K, pl.R, pl.S, is_deconv, pl.alpha, pl.NT, pl.NB, pl.NCC, pl.pair ? 2 : 1, G.data(),
-                              stream) != cudaSuccess)
+                              tag, static_cast<UTag*>(u), stream) != cudaSuccess)
     return I2CW_ECUDA;
   return I2CW_OK;
 }

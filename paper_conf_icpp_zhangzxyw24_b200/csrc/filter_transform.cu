@@ -22,8 +22,11 @@ struct GTable {
 
 __global__ void filter_transform_kernel(const float* __restrict__ w, float* __restrict__ u, int C, int K, int R,
                                         int S, int is_deconv, int alpha, int NT, int NB, int NCC, int halves,
-                                        GTable gt) {
+                                        GTable gt, UTag tag, UTag* tag_dst) {
   const int NKS = NCC * R;
+  // the 256-byte tag in front of U (checked by the _pretransformed calls), written here instead
+  // of by a separate host-to-device copy
+  if (tag_dst && blockIdx.x == 0 && threadIdx.x == 0) *tag_dst = tag;
   const size_t total = (size_t)NB * NKS * alpha * 2 * NT * 4;  // (nb, ks, idx, kc, n, e)
   for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < total; i += (size_t)gridDim.x * blockDim.x) {
     size_t t = i;
@@ -62,7 +65,7 @@ __global__ void filter_transform_kernel(const float* __restrict__ w, float* __re
 
 cudaError_t launch_filter_transform(const float* w, float* u, int C, int K, int R, int S, int is_deconv, int alpha,
                                     int NT, int NB, int NCC, int halves, const double* G /* alpha x S, internal order */,
-                                    cudaStream_t stream) {
+                                    const UTag& tag, UTag* tag_dst, cudaStream_t stream) {
   GTable gt;
   for (int i = 0; i < 16 * 9; ++i) gt.g[i] = 0.0;
   for (int i = 0; i < alpha; ++i)
@@ -71,7 +74,8 @@ cudaError_t launch_filter_transform(const float* w, float* u, int C, int K, int 
   int blocks = (int)((total + 255) / 256);
   if (blocks > 148 * 16) blocks = 148 * 16;
   if (blocks < 1) blocks = 1;
-  filter_transform_kernel<<<blocks, 256, 0, stream>>>(w, u, C, K, R, S, is_deconv, alpha, NT, NB, NCC, halves, gt);
+  filter_transform_kernel<<<blocks, 256, 0, stream>>>(w, u, C, K, R, S, is_deconv, alpha, NT, NB, NCC, halves, gt,
+                                                      tag, tag_dst);
   return cudaGetLastError();
 }
 
