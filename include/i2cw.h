@@ -24,7 +24,12 @@
  *    default stream) and the call returns without a host sync; kernel faults
  *    surface at the caller's next synchronisation.
  *  - The library keeps no global mutable state except a lazily created
- *    stream-ordered workspace pool (see i2cw_conv2d_nhwc).
+ *    stream-ordered workspace pool (see i2cw_conv2d_nhwc), a memo of launch plans
+ *    and transform tables (pure functions of the dimensions), and two copy streams
+ *    per device for i2cw_conv2d_nhwc_host.
+ *  - A conv/deconv call may enqueue a cudaMemsetAsync on part of y before its kernel
+ *    (the "split tail" of the persistent schedule, whose two Winograd passes both
+ *    reduce-add into y); results are bitwise deterministic run to run.
  *  - fp32 in / fp32 out. The per-point channel contraction runs on the tcgen05
  *    tensor cores in 3xTF32 (hi*hi + hi*lo + lo*hi), which keeps
  *    |y - y_exact| <= 1e-4 * sum|x|*|w| per element (BASELINE.json north_star).

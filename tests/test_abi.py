@@ -76,6 +76,14 @@ def test_planner_consistency(cfg):
     assert p["NB"] * p["NT"] >= K and p["NCC"] * 8 >= C
     assert p["smem_bytes"] <= 227 * 1024
     assert p["tile_blocks"] == -(-N // p["NI"]) * p["PB"] * p["SEGS"]
+    # work items (persistent schedule): whole units, then a split tail of T units as 2T
+    # one-pass items, only with 2 passes, no CTA pairs and 2T <= #CTAs (148 without a GPU)
+    units = (-(-p["tile_blocks"] // 2) if p["pair"] else p["tile_blocks"]) * p["NB"]
+    T = units - p["NFULL"]
+    assert 0 <= T and p["NITEMS"] == p["NFULL"] + 2 * T
+    if T:
+        G = 148
+        assert p["NPASS"] == 2 and not p["pair"] and 2 * T <= G and p["NFULL"] % G == 0
 
 
 def test_invalid_arguments_rejected_before_cuda():
