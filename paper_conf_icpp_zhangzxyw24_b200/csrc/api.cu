@@ -158,10 +158,11 @@ int make_plan_uncached(int N, int H, int W, int C, int K, int R, int S, int pad_
   pl.SEGS = cdiv(pl.T_r, pl.TS);
   // CTA pairs (clusters of 2, tcgen05.mma.cta_group::2 with M = 256, each CTA stages half of
   // U): halves the per-SM filter stream and B-operand reads but adds a cross-CTA relay per
-  // super-stage. Measured on B200 (profiles/r01d_pair_sweep.txt): +5..12% at NKS = C/8 * R >= 128
-  // (r9, cfg4 r5/r7, c512), -2..-18% below (cfg2, r2-r7, c64, c128). I2CW_PAIR=1/0 forces it.
+  // super-stage. Measured on B200 (profiles/r01d_pair_sweep.txt, profiles/r01i_pair_rule.txt):
+  // +5..12% at NKS = C/8 * R >= 128 (r8, r9, cfg4 r5/r7, c512) or >= 4 output-channel blocks
+  // (c256 +11%), -2..-18% otherwise (cfg2, r2-r7, c64, c128). I2CW_PAIR=1/0 forces it.
   static const int pair_env = [] { const char* e = getenv("I2CW_PAIR"); return e ? (e[0] == '1' ? 1 : 0) : -1; }();
-  pl.pair = pair_env >= 0 ? pair_env : (pl.NKS >= 128 ? 1 : 0);
+  pl.pair = pair_env >= 0 ? pair_env : ((pl.NKS >= 128 || pl.NB >= 4) ? 1 : 0);
   // DEBUG timing ablation (never set in production; results are wrong when non-zero)
   static const int ablate = [] { const char* e = getenv("I2CW_ABLATE"); return e ? atoi(e) : 0; }();
   pl.ablate = ablate;
