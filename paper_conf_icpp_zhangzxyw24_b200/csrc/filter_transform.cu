@@ -24,6 +24,9 @@ __global__ void filter_transform_kernel(const float* __restrict__ w, float* __re
                                         int S, int is_deconv, int alpha, int NT, int NB, int NCC, int halves,
                                         GTable gt, UTag tag, UTag* tag_dst) {
   const int NKS = NCC * R;
+  // let a programmatically dependent fused kernel start its prologue now (it waits with
+  // griddepcontrol.wait before reading U, which covers this grid's completion)
+  asm volatile("griddepcontrol.launch_dependents;");
   // the 256-byte tag in front of U (checked by the _pretransformed calls), written here instead
   // of by a separate host-to-device copy
   if (tag_dst && blockIdx.x == 0 && threadIdx.x == 0) *tag_dst = tag;

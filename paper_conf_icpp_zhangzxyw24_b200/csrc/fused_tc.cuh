@@ -490,6 +490,9 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
     if (lane32 == 0) {
       tma_prefetch_desc(&xmap);
       tma_prefetch_desc(&ymap);
+      // programmatic dependent launch: the prologue above overlapped the previous kernel;
+      // its results (x, U) are visible only after this wait
+      asm volatile("griddepcontrol.wait;" ::: "memory");
       int ist = 0, iph = 0, first = 1;  // slot, round parity, still in the first round
       for (int it = unit0; it < NITEMS; it += ustride) {
       const Item I = item_at(it);
@@ -516,6 +519,7 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
   } else if (warp == UPROD_WARP) {
     // ================= U (transformed filter) super-slot ring =================
     if (lane32 == 0) {
+      asm volatile("griddepcontrol.wait;" ::: "memory");  // U written by the previous kernel
       const size_t kstride = (size_t)A * 2 * NT * 8;  // floats per k-step (both layouts)
       int us = 0, uph = 0, first = 1;
       for (int it = unit0; it < NITEMS; it += ustride) {
@@ -681,17 +685,30 @@ static cudaError_t launch_tc_t(const CUtensorMap& xmap, const CUtensorMap& ymap,
     cfg.blockDim = dim3(Cfg::NTHREADS);
     cfg.dynamicSmemBytes = pl.smem_bytes;
     cfg.stream = stream;
-    cudaLaunchAttribute attr[1];
+    cudaLaunchAttribute attr[2];
     attr[0].id = cudaLaunchAttributeClusterDimension;
     attr[0].val.clusterDim.x = 2;
     attr[0].val.clusterDim.y = 1;
     attr[0].val.clusterDim.z = 1;
+    attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[1].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 2;
+    e = cudaLaunchKernelEx(&cfg, kern, xmap, ymap, pl, u);
+    if (e != cudaSuccess) return e;
+  } else {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(persistent_ctas(pl.NITEMS, 1));
+    cfg.blockDim = dim3(Cfg::NTHREADS);
+    cfg.dynamicSmemBytes = pl.smem_bytes;
+    cfg.stream = stream;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;  // overlap the prologue
+    attr[0].val.programmaticStreamSerializationAllowed = 1;            // with the previous kernel
     cfg.attrs = attr;
     cfg.numAttrs = 1;
     e = cudaLaunchKernelEx(&cfg, kern, xmap, ymap, pl, u);
     if (e != cudaSuccess) return e;
-  } else {
-    kern<<<persistent_ctas(pl.NITEMS, 1), Cfg::NTHREADS, pl.smem_bytes, stream>>>(xmap, ymap, pl, u);
   }
   return cudaGetLastError();
 }
