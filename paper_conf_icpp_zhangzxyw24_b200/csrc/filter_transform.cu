@@ -21,7 +21,7 @@ struct GTable {
 };
 
 __global__ void filter_transform_kernel(const float* __restrict__ w, float* __restrict__ u, int C, int K, int R,
-                                        int S, int is_deconv, int alpha, int NT, int NB, int NCC, int halves,
+                                        int S, int is_deconv, int alpha, int NT, int NB, int NCC, int halves, int npg,
                                         GTable gt, UTag tag, UTag* tag_dst) {
   const int NKS = NCC * R;
   // let a programmatically dependent fused kernel start its prologue now (it waits with
@@ -30,38 +30,58 @@ __global__ void filter_transform_kernel(const float* __restrict__ w, float* __re
   // the 256-byte tag in front of U (checked by the _pretransformed calls), written here instead
   // of by a separate host-to-device copy
   if (tag_dst && blockIdx.x == 0 && threadIdx.x == 0) *tag_dst = tag;
-  const size_t total = (size_t)NB * NKS * alpha * 2 * NT * 4;  // (nb, ks, idx, kc, n, e)
+  // One thread per (point group, filter row segment (nb, ks, kc, n, e)): its S taps are read
+  // once and the alpha / npg points of its group are produced from registers (npg = 1 for
+  // large filters; small filters split the points over more threads to fill the GPU). The
+  // fastest thread index follows the filter's contiguous dimension (c for the KRSC conv
+  // filter, k for the CRSK deconv filter).
+  const size_t rows = (size_t)NB * NKS * 2 * NT * 4;
+  const size_t total = rows * npg;
+  const int ppg = alpha / npg;
   for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < total; i += (size_t)gridDim.x * blockDim.x) {
-    size_t t = i;
-    const int e = (int)(t % 4); t /= 4;
-    const int n = (int)(t % NT); t /= NT;
+    size_t t = i % rows;
+    const int g = (int)(i / rows);
+    int e, n;
+    if (is_deconv) {
+      n = (int)(t % NT); t /= NT;
+      e = (int)(t % 4); t /= 4;
+    } else {
+      e = (int)(t % 4); t /= 4;
+      n = (int)(t % NT); t /= NT;
+    }
     const int kc = (int)(t % 2); t /= 2;
-    const int idx = (int)(t % alpha); t /= alpha;
     const int ks = (int)(t % NKS); t /= NKS;
     const int nb = (int)t;
     const int cc = ks / R, fh = ks % R;
     const int k = nb * NT + n, c = cc * 8 + kc * 4 + e;
-    float hi = 0.f, lo = 0.f;
-    if (k < K && c < C) {
-      double acc = 0.0;
-      for (int s = 0; s < S; ++s) {
-        const float wv = is_deconv ? w[(((size_t)c * R + (R - 1 - fh)) * S + (S - 1 - s)) * K + k]
-                                   : w[(((size_t)k * R + fh) * S + s) * C + c];
-        acc += gt.g[idx * 9 + s] * (double)wv;
-      }
-      const float uv = (float)acc;
-      hi = tf32_rna(uv);
-      lo = tf32_rna(uv - hi);
+    const bool live = k < K && c < C;
+    double wv[9];
+#pragma unroll
+    for (int s = 0; s < 9; ++s) {
+      wv[s] = 0.0;
+      if (live && s < S)
+        wv[s] = (double)(is_deconv ? w[(((size_t)c * R + (R - 1 - fh)) * S + (S - 1 - s)) * K + k]
+                                   : w[(((size_t)k * R + fh) * S + s) * C + c]);
     }
-    if (halves == 2) {  // CTA-pair layout: [h][idx][hl][kc][n'][e] per (nb, ks)
-      const int hN = NT / 2, h = n / hN, n2 = n % hN;
-      const size_t base = u_offset_pair(NT, alpha, nb, NKS, ks, h, idx) + (size_t)kc * hN * 4 + (size_t)n2 * 4 + e;
-      u[base] = hi;
-      u[base + (size_t)hN * 8] = lo;
-    } else {
-      const size_t base = u_offset(NT, alpha, nb, NKS, ks, idx, 0) + (size_t)kc * NT * 4 + (size_t)n * 4 + e;
-      u[base] = hi;
-      u[base + (size_t)NT * 8] = lo;  // hl = 1 image follows the hl = 0 image
+    for (int idx = g * ppg; idx < (g + 1) * ppg; ++idx) {
+      double acc = 0.0;
+#pragma unroll
+      for (int s = 0; s < 9; ++s)
+        if (s < S) acc += gt.g[idx * 9 + s] * wv[s];
+      const float uv = (float)acc;
+      const float hi = tf32_rna(uv);
+      const float lo = tf32_rna(uv - hi);
+      if (halves == 2) {  // CTA-pair layout: [h][idx][hl][kc][n'][e] per (nb, ks)
+        const int hN = NT / 2, h = n / hN, n2 = n % hN;
+        const size_t base =
+            u_offset_pair(NT, alpha, nb, NKS, ks, h, idx) + (size_t)kc * hN * 4 + (size_t)n2 * 4 + e;
+        u[base] = hi;
+        u[base + (size_t)hN * 8] = lo;
+      } else {
+        const size_t base = u_offset(NT, alpha, nb, NKS, ks, idx, 0) + (size_t)kc * NT * 4 + (size_t)n * 4 + e;
+        u[base] = hi;
+        u[base + (size_t)NT * 8] = lo;  // hl = 1 image follows the hl = 0 image
+      }
     }
   }
 }
@@ -73,11 +93,15 @@ cudaError_t launch_filter_transform(const float* w, float* u, int C, int K, int 
   for (int i = 0; i < 16 * 9; ++i) gt.g[i] = 0.0;
   for (int i = 0; i < alpha; ++i)
     for (int s = 0; s < S; ++s) gt.g[i * 9 + s] = G[i * S + s];
-  const size_t total = (size_t)NB * NCC * R * alpha * 2 * NT * 4;
+  const size_t rows = (size_t)NB * NCC * R * 2 * NT * 4;
+  // point groups: split the alpha points over threads until ~148 x 1024 threads are live
+  int npg = 1;
+  while (npg < alpha && alpha % (2 * npg) == 0 && rows * npg < (size_t)148 * 1024) npg *= 2;
+  const size_t total = rows * npg;
   int blocks = (int)((total + 255) / 256);
   if (blocks > 148 * 16) blocks = 148 * 16;
   if (blocks < 1) blocks = 1;
-  filter_transform_kernel<<<blocks, 256, 0, stream>>>(w, u, C, K, R, S, is_deconv, alpha, NT, NB, NCC, halves, gt,
+  filter_transform_kernel<<<blocks, 256, 0, stream>>>(w, u, C, K, R, S, is_deconv, alpha, NT, NB, NCC, halves, npg, gt,
                                                       tag, tag_dst);
   return cudaGetLastError();
 }
