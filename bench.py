@@ -340,7 +340,8 @@ def main():
                          "frac_vs_ubench_tf32": achieved / TF32_UBENCH_TFLOPS,
                          "ubench_tf32_tflops": TF32_UBENCH_TFLOPS,
                          "filter_transform_ms": t_ft / args.steps * 1e3},
-            "gpu_launches": 2 * args.steps,
+            # filter transform + fused kernel, + the split-tail zeroing kernel when the plan has one
+            "gpu_launches": (3 if p["NITEMS"] != p["NFULL"] else 2) * args.steps,
             "clocks": clocks,
         }
         if e2e is not None:

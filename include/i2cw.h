@@ -27,9 +27,10 @@
  *    stream-ordered workspace pool (see i2cw_conv2d_nhwc), a memo of launch plans
  *    and transform tables (pure functions of the dimensions), and two copy streams
  *    per device for i2cw_conv2d_nhwc_host.
- *  - A conv/deconv call may enqueue a cudaMemsetAsync on part of y before its kernel
- *    (the "split tail" of the persistent schedule, whose two Winograd passes both
- *    reduce-add into y); results are bitwise deterministic run to run.
+ *  - A conv/deconv call may enqueue a small zeroing kernel on part of y before its
+ *    fused kernel (the "split tail" of the persistent schedule, whose two Winograd
+ *    passes both reduce-add into y); it is a programmatic dependent of the previous
+ *    kernel in the stream and writes only y. Results are bitwise deterministic.
  *  - fp32 in / fp32 out. The per-point channel contraction runs on the tcgen05
  *    tensor cores in 3xTF32 (hi*hi + hi*lo + lo*hi), which keeps
  *    |y - y_exact| <= 1e-4 * sum|x|*|w| per element (BASELINE.json north_star).

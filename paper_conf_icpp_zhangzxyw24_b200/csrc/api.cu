@@ -22,6 +22,7 @@ cudaError_t launch_filter_transform(const float* w, float* u, int C, int K, int 
                                     UTag* tag_dst, cudaStream_t stream);
 cudaError_t launch_fused_tc(const CUtensorMap& xmap, const CUtensorMap& ymap, const Plan& pl, const float* u,
                             cudaStream_t stream);
+cudaError_t launch_zero_tail(float* y, size_t count, cudaStream_t stream);
 cudaError_t launch_fused_simt(const Plan& pl, const float* x, const float* u, float* y, cudaStream_t stream);
 
 namespace {
@@ -455,7 +456,7 @@ int run_fused(const Plan& pl, const float* x, const void* u, float* y, cudaStrea
     const int tb0 = pl.NFULL / pl.NB;
     const size_t n0 = (size_t)(tb0 / pl.SEGS / pl.PB) * pl.NI;
     const size_t img = (size_t)pl.P * pl.Q * pl.K;
-    if (n0 < (size_t)pl.N && cudaMemsetAsync(y + n0 * img, 0, ((size_t)pl.N - n0) * img * sizeof(float), stream) != cudaSuccess)
+    if (n0 < (size_t)pl.N && launch_zero_tail(y + n0 * img, ((size_t)pl.N - n0) * img, stream) != cudaSuccess)
       return I2CW_ECUDA;
   }
   int rc = encode_x_map(pl, x, &map);

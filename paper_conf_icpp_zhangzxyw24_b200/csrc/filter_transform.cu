@@ -12,6 +12,9 @@
 //   deconv: w'(k, fh, s, c) = w[c][R-1-fh][S-1-s][k]              (w is [C][R][S][K])
 // G is applied in fp64 and rounded once to fp32 (the filter
 // transform's precision hardly matters); hi = tf32_rna(u), lo = tf32_rna(u - hi).
+#include <algorithm>
+#include <cstdint>
+
 #include "common.cuh"
 
 namespace i2cw {
@@ -104,6 +107,43 @@ cudaError_t launch_filter_transform(const float* w, float* u, int C, int K, int 
   filter_transform_kernel<<<blocks, 256, 0, stream>>>(w, u, C, K, R, S, is_deconv, alpha, NT, NB, NCC, halves, npg, gt,
                                                       tag, tag_dst);
   return cudaGetLastError();
+}
+
+// Split-tail pre-zeroing of y (DESIGN.md §6.2 "split tail"), as a kernel instead of a
+// cudaMemsetAsync: a memset node between the filter transform and the fused kernel would end
+// their programmatic-dependent-launch overlap. This kernel is itself launched as a programmatic
+// dependent of the filter transform (it does not read U, so it may run concurrently with it),
+// lets the fused kernel launch at once, and waits for the filter transform's grid before it
+// exits, so the fused kernel's griddepcontrol.wait (on this grid) still covers U.
+__global__ void zero_tail_kernel(float* __restrict__ y, size_t count) {
+  asm volatile("griddepcontrol.launch_dependents;");
+  const size_t tid = blockIdx.x * (size_t)blockDim.x + threadIdx.x, nth = (size_t)gridDim.x * blockDim.x;
+  size_t head = 0;
+  if ((reinterpret_cast<uintptr_t>(y) & 15) == 0) {
+    float4* y4 = reinterpret_cast<float4*>(y);
+    const size_t n4 = count / 4;
+    for (size_t i = tid; i < n4; i += nth) y4[i] = make_float4(0.f, 0.f, 0.f, 0.f);
+    head = n4 * 4;
+  }
+  for (size_t i = head + tid; i < count; i += nth) y[i] = 0.f;
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+}
+
+cudaError_t launch_zero_tail(float* y, size_t count, cudaStream_t stream) {
+  if (count == 0) return cudaSuccess;
+  size_t want = (count / 4 + 255) / 256;
+  const unsigned blocks = (unsigned)std::min<size_t>(std::max<size_t>(want, 1), 148 * 8);
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(blocks);
+  cfg.blockDim = dim3(256);
+  cfg.stream = stream;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  cudaError_t e = cudaLaunchKernelEx(&cfg, zero_tail_kernel, y, count);
+  return e != cudaSuccess ? e : cudaGetLastError();
 }
 
 }  // namespace i2cw
