@@ -595,7 +595,9 @@ int i2cw_conv2d_nhwc_host(int is_deconv, int N, int H, int W, int C, int K, int 
   // Pipelined over image chunks: the host->device copy of chunk c+1 and the device->host copy
   // of chunk c-1 run on two copy streams while chunk c computes on `stream` (PCIe is full
   // duplex; the copies, not the kernel, bound this call). The filter is transformed once.
-  const int nchunk = std::max(1, std::min(N, 8));
+  // I2CW_HOST_CHUNKS=<n> (experiments): chunk count; 8 measured best on cfg2
+  static const int chunks_env = [] { const char* e = getenv("I2CW_HOST_CHUNKS"); return e ? atoi(e) : 0; }();
+  const int nchunk = std::max(1, std::min(N, chunks_env > 0 ? chunks_env : 8));
   const size_t img_x = (size_t)H * W * C, img_y = (size_t)pl.P * pl.Q * K;
   const size_t xb = (size_t)N * img_x * 4, wb = (size_t)K * R * S * C * 4, yb = (size_t)N * img_y * 4;
   static cudaStream_t s_in[64] = {}, s_out[64] = {};
