@@ -120,25 +120,56 @@ class ClockSampler:
                 "samples": len(self.samples)}
 
 
-def cpu_oracle_sample(cfg, budget_s=12.0, max_images=None):
-    """Time the fp64 oracle (y only) on a bounded sample of whole images of the workload."""
+def cpu_oracle_sample(cfg, budget_s=12.0, max_images=None, y_gpu=None, x_dev=None, w_dev=None):
+    """The fp64 oracle timed (y only) on a bounded sample of whole images of the workload, on the
+    host cores. With the GPU's own x / w / y it also verifies the timed run on that sample (max
+    |err| / sum|x||w| and the mean relative error, y and bound on the first image(s)), and runs
+    one image of the paper's U[1,2] accuracy setting through the GPU."""
+    import numpy as np
+    import torch
+
     import oracle
     from synthetic import make_w, make_x
     kind, N, H, W, C, K, R, S, ph, pw, _ = cfg
-    w = make_w(K, R, S, C) if kind == "conv" else make_w(C, R, S, K)
     f = oracle.conv2d_nhwc if kind == "conv" else oracle.deconv2d_nhwc
-    x1 = make_x(0, 1, H, W, C)
+    if x_dev is not None:
+        xs, w = x_dev[: min(N, x_dev.shape[0])].cpu(), w_dev.cpu()
+    else:
+        w = make_w(K, R, S, C) if kind == "conv" else make_w(C, R, S, K)
+        xs = make_x(0, 1, H, W, C)
     t0 = time.perf_counter()
-    f(x1, w, ph, pw, with_bound=False)
+    f(xs[:1], w, ph, pw, with_bound=False)
     t1 = time.perf_counter() - t0
-    n = max(1, min(N if max_images is None else max_images, int(budget_s / max(t1, 1e-6))))
-    x = make_x(0, n, H, W, C)
+    n = max(1, min(xs.shape[0] if max_images is None else max_images, int(budget_s / max(t1, 1e-6))))
+    if x_dev is None and n > 1:
+        xs = make_x(0, n, H, W, C)
     t0 = time.perf_counter()
-    f(x, w, ph, pw, with_bound=False)
+    f(xs[:n], w, ph, pw, with_bound=False)
     dt = time.perf_counter() - t0
-    return {"value": direct_flops(cfg, n) / dt / 1e12, "unit": "TFLOPS", "cores": oracle.num_threads(),
-            "kind": "oracle",
-            "sample": f"{n} of {N} images of {cfg[-1]} (plain fp64 C oracle, y only), {dt:.2f} s"}
+    out = {"value": direct_flops(cfg, n) / dt / 1e12, "unit": "TFLOPS", "cores": oracle.num_threads(),
+           "kind": "oracle",
+           "sample": f"{n} of {N} images of {cfg[-1]} (plain fp64 C oracle, y only), {dt:.2f} s"}
+    if y_gpu is not None:
+        nv = min(2, n)
+        yr, b = f(xs[:nv], w, ph, pw)
+        yg = y_gpu[:nv].double().cpu().numpy()
+        e = np.abs(yg - yr)
+        nz = b > 0
+        out["verify"] = {"images": nv, "max_err_over_bound": float(np.max(e[nz] / b[nz])),
+                         "mean_rel_err": float(np.mean(e[nz] / np.maximum(np.abs(yr[nz]), 1e-30))),
+                         "what": "the timed run's y for these images vs the fp64 oracle (bound 1e-4)"}
+        import paper_conf_icpp_zhangzxyw24_b200 as i2cw
+        x12 = make_x(0, 1, H, W, C, 1.0, 2.0)
+        w12 = (make_w(K, R, S, C, 1.0, 2.0) if kind == "conv" else make_w(C, R, S, K, 1.0, 2.0))
+        g = (i2cw.conv2d_nhwc if kind == "conv" else i2cw.deconv2d_nhwc)(x12.to(x_dev.device), w12.to(x_dev.device),
+                                                                          ph, pw)
+        torch.cuda.synchronize()
+        yr, b = f(x12, w12, ph, pw)
+        e = np.abs(g.double().cpu().numpy() - yr)
+        out["accuracy_u12"] = {"images": 1, "mean_rel_err": float(np.mean(e / np.abs(yr))),
+                               "max_err_over_bound": float(np.max(e / b)),
+                               "what": "paper's Table 3 metric: U[1,2] inputs, mean |err|/|y| vs fp64"}
+    return out
 
 
 def run_reference(args, cfg):
@@ -187,6 +218,10 @@ def main():
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     ap.add_argument("--no-e2e", action="store_true", help="skip the host-buffer end-to-end leg")
     ap.add_argument("--e2e-steps", type=int, default=10)
+    ap.add_argument("--scaling", default="strong", choices=["strong", "weak"],
+                    help="strong: split the config's batch over the ranks (default); weak: N images per rank")
+    ap.add_argument("--no-sweep", action="store_true", help="skip the in-run r=2..9 sweep sub-object")
+    ap.add_argument("--no-peak", action="store_true", help="skip the cuBLAS TF32 peak measurement")
     args = ap.parse_args()
     if args.warmup < 3:
         raise SystemExit("--warmup must be >= 3")
@@ -199,7 +234,7 @@ def main():
     import torch.distributed as dist
 
     import paper_conf_icpp_zhangzxyw24_b200 as i2cw
-    from paper_conf_icpp_zhangzxyw24_b200.shard import max_over_ranks
+    from paper_conf_icpp_zhangzxyw24_b200.shard import gather_rows, max_over_ranks, shard_range
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -212,70 +247,119 @@ def main():
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
         dist.init_process_group("nccl", device_id=dev)
 
-    kind, N, H, W, C, K, R, S, ph, pw, desc = cfg
+    kind, N_cfg, H, W, C, K, R, S, ph, pw, desc = cfg
     P, Q = out_hw(kind, H, W, R, S, ph, pw)
     is_deconv = kind == "deconv"
-    # per-GPU batch fixed (weak scaling); images of rank r are global images r*N .. r*N+N-1
-    g = torch.Generator(device=dev).manual_seed(1000 + rank)
-    x = torch.rand((N, H, W, C), generator=g, device=dev).mul_(2).sub_(1)
-    g.manual_seed(7)
+    # Strong scaling (default): the config's batch N is split over the ranks,
+    # rank r owns global images [n0, n1). --scaling weak keeps N images per rank instead.
+    if args.scaling == "strong":
+        n0, n1 = shard_range(N_cfg, world, rank)
+        N_job = N_cfg
+    else:
+        n0, n1 = rank * N_cfg, (rank + 1) * N_cfg
+        N_job = N_cfg * world
+    N = n1 - n0
+    x = make_x_device(n0, n1, H, W, C, dev)
+    g = torch.Generator(device=dev).manual_seed(7)
     w = torch.rand((K, R, S, C) if not is_deconv else (C, R, S, K), generator=g, device=dev).mul_(2).sub_(1)
     y = torch.empty((N, P, Q, K), device=dev)
-    u = torch.empty(i2cw.filter_bytes(C, K, R, S), dtype=torch.uint8, device=dev)
+    u = torch.empty(i2cw.filter_bytes(K, C, R, S), dtype=torch.uint8, device=dev)
     flush = torch.empty(64 * 1024 * 1024, dtype=torch.float32, device=dev)  # 256 MiB > 126 MB L2
     stream = torch.cuda.current_stream()
     L = i2cw.lib()
     sp = stream.cuda_stream
+    conv_fn = L.i2cw_deconv2d_nhwc if is_deconv else L.i2cw_conv2d_nhwc
     conv_pre = L.i2cw_deconv2d_nhwc_pretransformed if is_deconv else L.i2cw_conv2d_nhwc_pretransformed
 
-    def step():
-        rc = L.i2cw_filter_transform(C, K, R, S, int(is_deconv), w.data_ptr(), u.data_ptr(), sp)
+    def check(fn, rc):
         if rc:
-            raise i2cw.I2CWError("i2cw_filter_transform", rc)
+            raise i2cw.I2CWError(fn, rc)
+
+    def step():  # the public one-shot call: filter transform + fused kernel (+ split-tail zeroing)
+        check("conv", conv_fn(N, H, W, C, K, R, S, ph, pw, x.data_ptr(), w.data_ptr(), y.data_ptr(), sp))
+
+    def step_split(ev_mid):  # the same two launches through the '*' API, an event between them
+        check("i2cw_filter_transform", L.i2cw_filter_transform(K, C, R, S, int(is_deconv), w.data_ptr(),
+                                                               u.data_ptr(), sp))
         if ev_mid is not None:
             ev_mid.record(stream)
-        rc = conv_pre(N, H, W, C, K, R, S, ph, pw, x.data_ptr(), u.data_ptr(), y.data_ptr(), sp)
-        if rc:
-            raise i2cw.I2CWError("i2cw_conv2d_nhwc_pretransformed", rc)
+        check("pretransformed", conv_pre(N, H, W, C, K, R, S, ph, pw, x.data_ptr(), u.data_ptr(), y.data_ptr(), sp))
 
-    # warm-up (also validates the call path)
+    def timed(fn, steps, flush_l2=True):
+        """Sum of per-step CUDA-event times (s) over `steps` steps, L2 flushed before each."""
+        ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
+        for a, b in ev:
+            if flush_l2:
+                flush.zero_()
+            a.record(stream)
+            fn()
+            b.record(stream)
+        torch.cuda.synchronize()
+        return sum(a.elapsed_time(b) for a, b in ev) / 1e3
+
     for _ in range(args.warmup):
         flush.zero_()
-        ev_mid = torch.cuda.Event(enable_timing=True)
         step()
+    step_split(None)
     torch.cuda.synchronize()
 
-    evs = [[torch.cuda.Event(enable_timing=True) for _ in range(3)] for _ in range(args.steps)]
     sampler = ClockSampler(local)
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
     with sampler:
-        for i in range(args.steps):
-            flush.zero_()
-            e0, _, e2 = evs[i]
-            ev_mid = None  # no event between the two launches: it would break their PDL overlap
-            e0.record(stream)
-            step()
-            e2.record(stream)
+        t_total = timed(step, args.steps)                        # THE timed region: exactly K steps
         torch.cuda.synchronize()
-    if world > 1:
-        dist.barrier()
+        if world > 1:
+            dist.barrier()
+        # BASELINE.md protocol beside it: >= 100 back-to-back calls (inputs > L2, no flush),
+        # median of 5 repeats; also keeps the clock sampler busy for long enough
+        nb2b = max(100, args.steps)
+        b2b = []
+        for _ in range(5):
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            for _ in range(nb2b):
+                step()
+            b.record(stream)
+            torch.cuda.synchronize()
+            b2b.append(a.elapsed_time(b) / 1e3 / nb2b)
     torch.cuda.synchronize()
-    t_total = sum(e[0].elapsed_time(e[2]) for e in evs) / 1e3        # s, K steps
-    # attribution pass (for the roofline): the same K steps again with an event between the
-    # filter transform and the fused kernel, so each launch is timed on its own stream
-    torch.cuda.synchronize()
-    for i in range(args.steps):
+    # attribution pass: an event between the filter transform and the fused kernel
+    ev3 = [[torch.cuda.Event(enable_timing=True) for _ in range(3)] for _ in range(args.steps)]
+    for e0, e1, e2 in ev3:
         flush.zero_()
-        e0, ev_mid, e2 = evs[i]
         e0.record(stream)
-        step()
+        step_split(e1)
         e2.record(stream)
     torch.cuda.synchronize()
-    t_fused = sum(e[1].elapsed_time(e[2]) for e in evs) / 1e3
-    t_ft = sum(e[0].elapsed_time(e[1]) for e in evs) / 1e3
-    t_total, t_fused, t_ft = max_over_ranks([t_total, t_fused, t_ft], device=dev)  # NCCL MAX (world > 1)
+    t_ft = sum(e0.elapsed_time(e1) for e0, e1, _ in ev3) / 1e3
+    t_fused = sum(e1.elapsed_time(e2) for _, e1, e2 in ev3) / 1e3
+    # the paper's '*' number (PAPER.md:3951-3952): pre-transformed filter, fused kernel only
+    t_star = timed(lambda: check("pretransformed", conv_pre(N, H, W, C, K, R, S, ph, pw, x.data_ptr(), u.data_ptr(),
+                                                            y.data_ptr(), sp)), args.steps)
+    t_b2b = statistics.median(b2b)
+    t_total, t_fused, t_ft, t_star, t_b2b = max_over_ranks([t_total, t_fused, t_ft, t_star, t_b2b], device=dev)
+
+    # output sanity: every element finite (the timed runs wrote y)
+    finite = bool(torch.isfinite(y).all())
+    ok_all = max_over_ranks([0.0 if finite else 1.0], device=dev)[0] == 0.0
+    # sharding check (world > 1): NCCL all_gather of every rank's y to rank 0, compared with one
+    # single-GPU call over the whole batch on rank 0 (each side is oracle-verified by the -m gpu
+    # tests; this checks that every image was computed exactly once and lands in place)
+    shard_check = None
+    if world > 1 and args.scaling == "strong":
+        y_all = gather_rows(y)
+        if rank == 0:
+            x_full = make_x_device(0, N_cfg, H, W, C, dev)
+            f = i2cw.deconv2d_nhwc if is_deconv else i2cw.conv2d_nhwc
+            y_one = f(x_full, w, ph, pw)
+            bnd = f(x_full.abs(), w.abs(), ph, pw)
+            r = float(((y_all - y_one).abs() / bnd.clamp_min(1e-30)).max())
+            shard_check = {"images": N_cfg, "max_diff_over_bound": r, "ok": r <= 2e-4,
+                           "how": "NCCL all_gather of the shards vs one single-GPU call on rank 0"}
+            del x_full, y_one, bnd
+        del y_all
 
     # end-to-end through the public host-buffer call (H2D x, w + conv + D2H y every step)
     e2e = None
@@ -295,62 +379,184 @@ def main():
         eb.record(stream)
         torch.cuda.synchronize()
         te = max_over_ranks([ea.elapsed_time(eb) / 1e3], device=dev)[0]
-        e2e = {"value": direct_flops(cfg) * world * args.e2e_steps / te / 1e12, "unit": "TFLOPS",
-               "h2d_bytes_per_step": (x.numel() + w.numel()) * 4, "d2h_bytes_per_step": y.numel() * 4,
+        e2e = {"value": direct_flops(cfg, N_job) * args.e2e_steps / te / 1e12, "unit": "TFLOPS",
+               "h2d_bytes_per_step": (x.numel() + w.numel()) * 4 * world, "d2h_bytes_per_step": y.numel() * 4 * world,
                "steps": args.e2e_steps, "api": "i2cw_conv2d_nhwc_host (pinned host buffers)"}
 
     clocks = sampler.summary()
+    sweep = None
+    if world == 1 and not args.no_sweep and args.config == "cfg2":
+        sweep = run_sweep(i2cw, dev, flush)
     if rank == 0:
         pk, pk_src = load_peaks()
         p = i2cw.debug_plan(kind, N, H, W, C, K, R, S, ph, pw)
-        m, alpha = p["m"], p["alpha"]
-        # algorithmic tensor work of the fused kernel per launch: 3xTF32,
-        # fractional tiles per output row: F_tc = 3 * 2 * alpha * N * P * (Q/m) * K * R * C
-        f_tc = 3 * 2 * alpha * N * P * (Q / m) * K * R * C
-        t_fused_launch = t_fused / args.steps
-        tf32_peak = pk["bf16_tflops"] * 0.5  # tf32 dense = bf16 dense / 2 (nominal ratio)
-        achieved = f_tc / t_fused_launch / 1e12
-        # algorithmic HBM bytes of the fused kernel: x read once, y written once, U read once
-        hbm_bytes = 4 * (N * H * W * C + N * P * Q * K) + (i2cw.filter_bytes(C, K, R, S) - 256)
-        traffic = None
-        tpath = os.path.join(ROOT, "profiles", "traffic.json")
-        if os.path.exists(tpath):
-            try:
-                traffic = json.load(open(tpath)).get(args.config)
-            except Exception:
-                traffic = None
-        value = direct_flops(cfg) * world * args.steps / t_total / 1e12
+        rf = roofline(i2cw, cfg, N, p, t_fused / args.steps, pk, pk_src)
+        rf["traffic"] = load_traffic(args.config)
+        rf["filter_transform_ms"] = t_ft / args.steps * 1e3
+        tf32 = measure_tf32_peak(dev) if not args.no_peak else None
+        if tf32:
+            rf["tf32_cublas_tflops"] = tf32
+            rf["frac_vs_tf32_cublas"] = rf["achieved"] / tf32
+        value = direct_flops(cfg, N_job) * args.steps / t_total / 1e12
         line = {
             "metric": METRIC, "value": value, "unit": "TFLOPS", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": t_total / args.steps * 1e3, "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "f32 (3xTF32 tcgen05 contraction)",
+            "scaling": args.scaling, "vs_baseline": None, "dtype": "f32 (3xTF32 tcgen05 contraction)",
             "data": "synthetic",
-            "config": {"workload": desc, "name": args.config, "per_gpu_batch": N, "global_batch": N * world,
-                       "parallelism": f"batch-sharded x{world}, no collective in the timed region",
-                       "F(m,r)": f"F({m},{S}) alpha={alpha}", "l2": "flushed (256 MiB memset) before every step",
-                       "step": "i2cw_filter_transform + i2cw_conv2d_nhwc_pretransformed (C ABI)"},
-            "roofline": {"bound": "tensor", "achieved": achieved, "peak": tf32_peak, "unit": "TFLOP/s",
-                         "frac": achieved / tf32_peak, "traffic": traffic,
-                         "kernel": "fused_tc_kernel", "kernel_ms": t_fused_launch * 1e3,
-                         "work": "3xTF32 UMMA flops 6*alpha*N*P*(Q/m)*K*R*C per launch",
-                         "peak_src": f"{pk_src}: bf16_tflops {pk['bf16_tflops']} x 0.5 (tf32/bf16 nominal)",
-                         "hbm_frac": hbm_bytes / t_fused_launch / 1e9 / pk["hbm_gbs"],
-                         # transparency: the tf32 UMMA throughput our own microbenchmark reaches
-                         # (tools/mma_bench.cu, N = 256, 1.965 GHz) is above the nominal-ratio peak
-                         "frac_vs_ubench_tf32": achieved / TF32_UBENCH_TFLOPS,
-                         "ubench_tf32_tflops": TF32_UBENCH_TFLOPS,
-                         "filter_transform_ms": t_ft / args.steps * 1e3},
-            # filter transform + fused kernel, + the split-tail zeroing kernel when the plan has one
-            "gpu_launches": (3 if p["NITEMS"] != p["NFULL"] else 2) * args.steps,
+            "config": {"workload": desc, "name": args.config, "global_batch": N_job,
+                       "per_gpu_batch": N if args.scaling == "weak" else f"{N_cfg // world}-{-(-N_cfg // world)}",
+                       "parallelism": f"batch-sharded x{world} (shard_range), no collective in the timed region",
+                       "F(m,r)": f"F({p['m']},{S}) alpha={p['alpha']}", "l2": "flushed (256 MiB memset) before every step",
+                       "inputs": "x[n] ~ U[-1,1) seeded 1000+n per global image n (on device), w ~ U[-1,1) seed 7",
+                       "step": f"i2cw_{'de' if is_deconv else ''}conv2d_nhwc (C ABI one-shot call: filter transform + fused kernel)"},
+            "roofline": rf,
+            "protocol_b2b": {"value": direct_flops(cfg, N_job) / t_b2b / 1e12, "unit": "TFLOPS", "calls": nb2b,
+                             "repeats": 5, "stat": "median of 5 repeats, max over ranks",
+                             "note": "BASELINE.md protocol: back-to-back one-shot calls, no L2 flush (inputs > L2)"},
+            "star": {"value": direct_flops(cfg, N_job) * args.steps / t_star / 1e12, "unit": "TFLOPS",
+                     "ms": t_star / args.steps * 1e3,
+                     "what": "pre-transformed filter (the paper's '*', PAPER.md:3951-3952): fused kernel only"},
+            # one-shot call = filter transform + one fused launch per K-chunk (+ split-tail zeroing)
+            "gpu_launches": (1 + p["NKC"] + (1 if p["NITEMS"] != p["NFULL"] else 0)) * args.steps,
+            "outputs_finite": ok_all,
             "clocks": clocks,
         }
+        if shard_check is not None:
+            line["shard_check"] = shard_check
         if e2e is not None:
             line["e2e"] = e2e
+        if sweep is not None:
+            line["sweep"] = sweep
         if world == 1 and not args.no_cpu:
-            line["cpu_baseline"] = cpu_oracle_sample(cfg)
+            line["cpu_baseline"] = cpu_oracle_sample(cfg, y_gpu=y, x_dev=x, w_dev=w)
         print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()
+
+
+def make_x_device(n0, n1, H, W, C, dev):
+    """Global images n0..n1-1 drawn ON the device, one generator seed (1000 + n) per image, so a
+    sharded run sees exactly the images of the unsharded one."""
+    import torch
+    x = torch.empty((n1 - n0, H, W, C), device=dev)
+    g = torch.Generator(device=dev)
+    for i, n in enumerate(range(n0, n1)):
+        g.manual_seed(1000 + n)
+        x[i] = torch.rand((H, W, C), generator=g, device=dev).mul_(2).sub_(1)
+    return x
+
+
+def roofline(i2cw, cfg, N, p, t_launch, pk, pk_src):
+    """Roofline object of the fused kernel; t_launch = its CUDA-event time."""
+    kind, _, H, W, C, K, R, S, ph, pw, _ = cfg
+    P, Q = out_hw(kind, H, W, R, S, ph, pw)
+    m, alpha = p["m"], p["alpha"]
+    # algorithmic tensor work per launch: 3xTF32 flops with fractional tiles per row
+    f_tc = 3 * 2 * alpha * N * P * (Q / m) * K * R * C
+    tf32_peak = pk["bf16_tflops"] * 0.5  # tf32 dense = bf16 dense / 2 (nominal ratio)
+    achieved = f_tc / t_launch / 1e12
+    hbm_bytes = 4 * (N * H * W * C + N * P * Q * K) + (i2cw.filter_bytes(K, C, R, S) - 256)
+    rf = {"bound": "tensor", "achieved": achieved, "peak": tf32_peak, "unit": "TFLOP/s",
+          "frac": achieved / tf32_peak, "kernel": "fused_tc_kernel", "kernel_ms": t_launch * 1e3,
+          "work": "3xTF32 UMMA flops 6*alpha*N*P*(Q/m)*K*R*C per launch",
+          "peak_src": f"{pk_src}: bf16_tflops {pk['bf16_tflops']} x 0.5 (tf32/bf16 nominal)",
+          "hbm_frac": hbm_bytes / t_launch / 1e9 / pk["hbm_gbs"],
+          "frac_vs_ubench_tf32": achieved / TF32_UBENCH_TFLOPS, "ubench_tf32_tflops": TF32_UBENCH_TFLOPS}
+    # anti-gaming rule (SURVEY.md §8(d)): the same time against the default-table (m, alpha) of §8(a)
+    dm, da = DEFAULT_TABLE[S]
+    if (dm, da) != (m, alpha):
+        f_def = 3 * 2 * da * N * P * (Q / dm) * K * R * C
+        rf["frac_default_table"] = f_def / t_launch / 1e12 / tf32_peak
+        rf["default_table"] = f"F({dm},{S}) alpha={da}"
+    return rf
+
+
+# SURVEY.md §8(a) default (m, alpha) per filter width (r = 8, 9: the paper's Gamma16)
+DEFAULT_TABLE = {2: (7, 8), 3: (6, 8), 4: (5, 8), 5: (4, 8), 6: (3, 8), 7: (2, 8), 8: (9, 16), 9: (8, 16)}
+
+
+def load_traffic(name):
+    tpath = os.path.join(ROOT, "profiles", "traffic.json")
+    try:
+        return json.load(open(tpath)).get(name)
+    except Exception:
+        return None
+
+
+def measure_tf32_peak(dev):
+    """cuBLAS fp32 GEMM with TF32 allowed, 8192^3, best of 10 (the MEASURED_PEAKS protocol)."""
+    import torch
+    try:
+        old = torch.backends.cuda.matmul.allow_tf32
+        torch.backends.cuda.matmul.allow_tf32 = True
+        a = torch.randn(8192, 8192, device=dev)
+        b = torch.randn(8192, 8192, device=dev)
+        c = a @ b
+        best = 1e9
+        for _ in range(10):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            torch.matmul(a, b, out=c)
+            e1.record()
+            torch.cuda.synchronize()
+            best = min(best, e0.elapsed_time(e1) / 1e3)
+        torch.backends.cuda.matmul.allow_tf32 = old
+        del a, b, c
+        return 2 * 8192 ** 3 / best / 1e12
+    except Exception:
+        return None
+
+
+SWEEP = ["cfg3-r2", "cfg3-r3", "cfg3-r4", "cfg3-r5", "cfg3-r6", "cfg3-r7", "cfg3-r8", "cfg3-r9", "cfg4-r5",
+         "cfg4-r7", "cfg5b-c64", "cfg5b-c512"]
+
+
+def run_sweep(i2cw, dev, flush, steps=10):
+    """The metric's r = 2..9 sweep (and cfg4 / cfg5b ends) in the same run: per config the
+    one-shot call, L2 flushed per step, 3 warm-ups; kernel-only time for the roofline."""
+    import torch
+    pk, pk_src = load_peaks()
+    L = i2cw.lib()
+    out = {}
+    for name in SWEEP:
+        cfg = CONFIGS[name]
+        kind, N, H, W, C, K, R, S, ph, pw, _ = cfg
+        P, Q = out_hw(kind, H, W, R, S, ph, pw)
+        dec = kind == "deconv"
+        x = make_x_device(0, N, H, W, C, dev)
+        g = torch.Generator(device=dev).manual_seed(7)
+        w = torch.rand((K, R, S, C) if not dec else (C, R, S, K), generator=g, device=dev).mul_(2).sub_(1)
+        y = torch.empty((N, P, Q, K), device=dev)
+        u = torch.empty(i2cw.filter_bytes(K, C, R, S), dtype=torch.uint8, device=dev)
+        sp = torch.cuda.current_stream().cuda_stream
+        fn = L.i2cw_deconv2d_nhwc if dec else L.i2cw_conv2d_nhwc
+        pre = L.i2cw_deconv2d_nhwc_pretransformed if dec else L.i2cw_conv2d_nhwc_pretransformed
+        L.i2cw_filter_transform(K, C, R, S, int(dec), w.data_ptr(), u.data_ptr(), sp)
+        ts, tk = 0.0, 0.0
+        for i in range(steps + 3):
+            flush.zero_()
+            e0, e1, e2 = (torch.cuda.Event(enable_timing=True) for _ in range(3))
+            e0.record()
+            rc = fn(N, H, W, C, K, R, S, ph, pw, x.data_ptr(), w.data_ptr(), y.data_ptr(), sp)
+            e1.record()
+            flush.zero_()
+            e3 = torch.cuda.Event(enable_timing=True)
+            e3.record()
+            rc |= pre(N, H, W, C, K, R, S, ph, pw, x.data_ptr(), u.data_ptr(), y.data_ptr(), sp)
+            e2.record()
+            torch.cuda.synchronize()
+            if rc:
+                raise i2cw.I2CWError(name, rc)
+            if i >= 3:
+                ts += e0.elapsed_time(e1) / 1e3
+                tk += e3.elapsed_time(e2) / 1e3
+        p = i2cw.debug_plan(kind, N, H, W, C, K, R, S, ph, pw)
+        rf = roofline(i2cw, cfg, N, p, tk / steps, pk, pk_src)
+        out[name] = {"value": direct_flops(cfg) * steps / ts / 1e12, "unit": "TFLOPS", "kernel_ms": rf["kernel_ms"],
+                     "frac": rf["frac"], "F(m,r)": f"F({p['m']},{S}) alpha={p['alpha']}",
+                     **({"frac_default_table": rf["frac_default_table"]} if "frac_default_table" in rf else {})}
+        del x, w, y, u
+    return out
 
 
 if __name__ == "__main__":

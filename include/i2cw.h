@@ -103,20 +103,59 @@ I2CW_API int i2cw_deconv2d_nhwc(int N, int H, int W, int C, int K, int R, int S,
                        const float* x, const float* w, float* y, i2cw_stream_t stream);
 
 /*
+ * 3D convolution (Im2col-Winograd "can be applied to ND convolution, by
+ * expanding Stage1 Im2col to ND, while remaining Stage2 unchanged"): the 1D F(m, S) Winograd
+ * runs along W exactly as in 2D; the K loop of the channel contraction runs over (c, depth tap
+ * t, filter row r).
+ *   x: [N][D][H][W][C] fp32, w: [K][T][R][S][C] fp32, y: [N][OD][P][Q][K] fp32,
+ *   y[n][od][p][q][k] = sum_{t<T,r<R,s<S,c<C} x[n][od-pad_d+t][p-pad_h+r][q-pad_w+s][c] * w[k][t][r][s][c]
+ *   OD = D + 2*pad_d - T + 1 (P, Q as in 2D), zero padding.
+ * i2cw_deconv3d_ndhwc: the unit-stride transposed 3D conv, w: [C][T][R][S][K],
+ *   y[n][od][p][q][k] = sum_{c,t,r,s} x[n][od+pad_d-t][p+pad_h-r][q+pad_w-s][c] * w[c][t][r][s][k],
+ *   OD = D + T - 1 - 2*pad_d (rotation of all three taps folded into the filter transform).
+ * Same conventions, errors and tolerance as the 2D calls; S in [2, 9], T, R >= 1; the 3D path
+ * always uses the default alpha = 8 (S <= 7) / 12 (S = 8, 9) transforms.
+ */
+I2CW_API int i2cw_conv3d_ndhwc(int N, int D, int H, int W, int C, int K, int T, int R, int S, int pad_d, int pad_h,
+                               int pad_w, const float* x, const float* w, float* y, i2cw_stream_t stream);
+I2CW_API int i2cw_deconv3d_ndhwc(int N, int D, int H, int W, int C, int K, int T, int R, int S, int pad_d, int pad_h,
+                                 int pad_w, const float* x, const float* w, float* y, i2cw_stream_t stream);
+
+/*
+ * NCHW layout adapters: PyTorch's default layouts.
+ *   i2cw_conv2d_nchw:   x [N][C][H][W], w [K][C][R][S] (OIHW), y [N][K][P][Q]
+ *   i2cw_deconv2d_nchw: x [N][C][H][W], w [C][K][R][S] (conv_transpose2d weight), y [N][K][P][Q]
+ * Same operation, padding, errors and tolerance as the NHWC calls. x, w are transposed to
+ * NHWC / KRSC (CRSK) into stream-ordered pool workspaces by a tiled transpose kernel, the NHWC
+ * path runs, and y is transposed back: one extra HBM read + write of x, w and y per call.
+ */
+I2CW_API int i2cw_conv2d_nchw(int N, int C, int H, int W, int K, int R, int S, int pad_h, int pad_w, const float* x,
+                              const float* w, float* y, i2cw_stream_t stream);
+I2CW_API int i2cw_deconv2d_nchw(int N, int C, int H, int W, int K, int R, int S, int pad_h, int pad_w,
+                                const float* x, const float* w, float* y, i2cw_stream_t stream);
+
+/*
  * Pre-transformed filters (the paper's '*' variant, PAPER.md:3951-3952, 4001-4004:
  * transform once, reuse across calls).
+ * Argument order (K, C, R, S) follows SURVEY.md §8(b): K = output channels, C = input
+ * channels of the call the filter is for (for a deconvolution: the K and C passed to
+ * i2cw_deconv2d_nhwc, i.e. w is [C][R][S][K]).
  * i2cw_filter_bytes: bytes of the transformed filter u for these dims
  *   (a 256-byte tag + 2 * alpha(S) * ceil(K/NT)*NT * R * ceil8(C) * 4), or 0 if the
- *   shape is unsupported. For a deconv pass (C, K) as the deconv's (input, output)
- *   channel counts, exactly as to i2cw_deconv2d_nhwc.
+ *   shape is unsupported.
  * i2cw_filter_transform: u = tag || U_hi/U_lo in the fused kernel's staging layout.
  *   is_deconv = 0: w is [K][R][S][C]; is_deconv = 1: w is [C][R][S][K].
  * The _pretransformed calls take u instead of w; a u produced for other dims or
- * the other is_deconv value is rejected with I2CW_EINVAL (the tag is read with a
- * small device-to-host copy on `stream`, which synchronises that stream).
+ * the other is_deconv value is rejected with I2CW_EINVAL. Validation: a host-side copy of
+ * the tag is kept for every u written by i2cw_filter_transform in this process; any other
+ * u (cloned, loaded, another process) or a registry mismatch has its device tag read with a
+ * small device-to-host copy on `stream` (which synchronises that stream). The fused kernel
+ * also checks the device tag itself and traps (a launch failure at the next sync) if it
+ * disagrees with the call, so a stale host copy can never run a mismatched u silently.
+ * u must stay alive and unmodified until the calls that read it have completed.
  */
-I2CW_API size_t i2cw_filter_bytes(int C, int K, int R, int S);
-I2CW_API int i2cw_filter_transform(int C, int K, int R, int S, int is_deconv, const float* w, void* u,
+I2CW_API size_t i2cw_filter_bytes(int K, int C, int R, int S);
+I2CW_API int i2cw_filter_transform(int K, int C, int R, int S, int is_deconv, const float* w, void* u,
                           i2cw_stream_t stream);
 I2CW_API int i2cw_conv2d_nhwc_pretransformed(int N, int H, int W, int C, int K, int R, int S, int pad_h, int pad_w,
                                     const float* x, const void* u, float* y, i2cw_stream_t stream);

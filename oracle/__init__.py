@@ -32,11 +32,11 @@ _lib = None
 
 
 def build(force: bool = False) -> str:
-    """Compile direct_conv.c with gcc -O2 -fopenmp (plain C, no vector tricks)."""
-    src = os.path.join(_HERE, "direct_conv.c")
-    if force or not os.path.exists(_LIB_PATH) or os.path.getmtime(_LIB_PATH) < os.path.getmtime(src):
+    """Compile direct_conv.c (2D) and direct_conv3d.c (3D) with gcc -O2 -fopenmp (plain C)."""
+    srcs = [os.path.join(_HERE, f) for f in ("direct_conv.c", "direct_conv3d.c")]
+    if force or not os.path.exists(_LIB_PATH) or os.path.getmtime(_LIB_PATH) < max(map(os.path.getmtime, srcs)):
         tmp = _LIB_PATH + f".tmp{os.getpid()}"
-        subprocess.check_call(["gcc", "-O2", "-fopenmp", "-fPIC", "-shared", "-o", tmp, src, "-lm"])
+        subprocess.check_call(["gcc", "-O2", "-fopenmp", "-fPIC", "-shared", "-o", tmp, *srcs, "-lm"])
         os.replace(tmp, _LIB_PATH)
     return _LIB_PATH
 
@@ -54,6 +54,10 @@ def _load():
         for name in ("oracle_conv2d_nhwc_f64_points", "oracle_deconv2d_nhwc_f64_points"):
             f = getattr(lib, name)
             f.argtypes = [I] * 9 + [P, P, L, P, P, P]
+            f.restype = I
+        for name in ("oracle_conv3d_ndhwc_f64", "oracle_deconv3d_ndhwc_f64"):
+            f = getattr(lib, name)
+            f.argtypes = [I] * 12 + [P, P, P, P]
             f.restype = I
         lib.oracle_num_threads.restype = I
         _lib = lib
@@ -131,6 +135,62 @@ def points(kind, x, w, pad_h, pad_w, idx):
     if rc != 0:
         raise ValueError("oracle: invalid shape or index")
     return y, b
+
+
+def _conv3d(kind, x, w, pd, ph, pw, with_bound):
+    x, w = _as_f32(x), _as_f32(w)
+    N, D, H, W, C = x.shape
+    if kind == "conv":
+        K, T, R, S, C2 = w.shape
+        shp = (N, D + 2 * pd - T + 1, H + 2 * ph - R + 1, W + 2 * pw - S + 1, K)
+        f = _load().oracle_conv3d_ndhwc_f64
+    else:
+        C2, T, R, S, K = w.shape
+        shp = (N, D + T - 1 - 2 * pd, H + R - 1 - 2 * ph, W + S - 1 - 2 * pw, K)
+        f = _load().oracle_deconv3d_ndhwc_f64
+    assert C == C2
+    y = np.empty(shp, np.float64)
+    b = np.empty(shp, np.float64) if with_bound else None
+    rc = f(N, D, H, W, C, K, T, R, S, pd, ph, pw, x.ctypes.data, w.ctypes.data, y.ctypes.data,
+           b.ctypes.data if b is not None else None)
+    if rc != 0:
+        raise ValueError("oracle: invalid shape")
+    return (y, b) if with_bound else y
+
+
+def conv3d_ndhwc(x, w, pad_d, pad_h, pad_w, with_bound=True):
+    """3D conv: x [N,D,H,W,C], w [K,T,R,S,C] fp32 -> (y, B) fp64 [N,OD,P,Q,K]."""
+    return _conv3d("conv", x, w, pad_d, pad_h, pad_w, with_bound)
+
+
+def deconv3d_ndhwc(x, w, pad_d, pad_h, pad_w, with_bound=True):
+    """3D transposed conv: x [N,D,H,W,C], w [C,T,R,S,K] fp32 -> (y, B) fp64 [N,OD,P,Q,K]."""
+    return _conv3d("deconv", x, w, pad_d, pad_h, pad_w, with_bound)
+
+
+def brute_conv3d_int(x, w, pd, ph, pw):
+    """Exact-integer 3D conv on Python ints (tiny shapes): x [N,D,H,W,C], w [K,T,R,S,C]."""
+    x = [[[[[int(v) for v in c] for c in row] for row in plane] for plane in img] for img in np.asarray(x)]
+    w = np.asarray(w).astype(np.int64)
+    N, D, H, W, C = len(x), len(x[0]), len(x[0][0]), len(x[0][0][0]), len(x[0][0][0][0])
+    K, T, R, S, _ = w.shape
+    OD, P, Q = D + 2 * pd - T + 1, H + 2 * ph - R + 1, W + 2 * pw - S + 1
+    y = np.zeros((N, OD, P, Q, K), dtype=object)
+    for n in range(N):
+        for d in range(OD):
+            for p in range(P):
+                for q in range(Q):
+                    for k in range(K):
+                        acc = 0
+                        for t in range(T):
+                            for r in range(R):
+                                for s in range(S):
+                                    i, j, l = d - pd + t, p - ph + r, q - pw + s
+                                    if 0 <= i < D and 0 <= j < H and 0 <= l < W:
+                                        for c in range(C):
+                                            acc += x[n][i][j][l][c] * int(w[k, t, r, s, c])
+                        y[n, d, p, q, k] = acc
+    return y
 
 
 # ---------------------------------------------------------------------------

@@ -25,6 +25,7 @@ PUBLIC_SYMBOLS = (
     "i2cw_status_string", "i2cw_version", "i2cw_conv2d_nhwc", "i2cw_deconv2d_nhwc", "i2cw_filter_bytes",
     "i2cw_filter_transform", "i2cw_conv2d_nhwc_pretransformed", "i2cw_deconv2d_nhwc_pretransformed",
     "i2cw_conv2d_nhwc_host", "i2cw_set_device", "i2cw_plan", "i2cw_transform_matrices_rational",
+    "i2cw_conv3d_ndhwc", "i2cw_deconv3d_ndhwc", "i2cw_conv2d_nchw", "i2cw_deconv2d_nchw",
 )
 
 
@@ -50,6 +51,14 @@ def lib():
             f = getattr(L, name)
             f.argtypes = [I] * 9 + [P, P, P, P]
             f.restype = I
+        for name in ("i2cw_conv2d_nchw", "i2cw_deconv2d_nchw"):
+            f = getattr(L, name)
+            f.argtypes = [I] * 9 + [P, P, P, P]
+            f.restype = I
+        for name in ("i2cw_conv3d_ndhwc", "i2cw_deconv3d_ndhwc"):
+            f = getattr(L, name)
+            f.argtypes = [I] * 12 + [P, P, P, P]
+            f.restype = I
         L.i2cw_filter_bytes.argtypes = [I] * 4
         L.i2cw_filter_bytes.restype = S
         L.i2cw_filter_transform.argtypes = [I] * 5 + [P, P, P]
@@ -66,6 +75,9 @@ def lib():
         L.i2cw_debug_conv_simt.restype = I
         L.i2cw_debug_plan.argtypes = [I] * 10 + [P]
         L.i2cw_debug_plan.restype = I
+        if hasattr(L, "i2cw_debug_set_kchunk"):  # test hook (absent from older experiment builds)
+            L.i2cw_debug_set_kchunk.argtypes = [I]
+            L.i2cw_debug_set_kchunk.restype = I
         _lib = L
     return _lib
 
@@ -91,6 +103,18 @@ def _check_tensor(t, name):
         raise ValueError(f"{name} must be a contiguous fp32 CUDA tensor")
 
 
+def _out(out, shp, like):
+    """The output tensor: a new one, or the caller's `out` after checking that the kernels may
+    write shp's elements into it (the TMA maps and the zeroing kernel use the plan's sizes)."""
+    import torch
+    if out is None:
+        return torch.empty(shp, dtype=torch.float32, device=like.device)
+    _check_tensor(out, "out")
+    if tuple(out.shape) != tuple(shp) or out.device != like.device:
+        raise ValueError(f"out must have shape {tuple(shp)} on {like.device}, got {tuple(out.shape)} on {out.device}")
+    return out
+
+
 def out_shape(kind, N, H, W, K, R, S, pad_h, pad_w):
     if kind == "conv":
         return (N, H + 2 * pad_h - R + 1, W + 2 * pad_w - S + 1, K)
@@ -105,9 +129,9 @@ def conv2d_nhwc(x, w, pad_h, pad_w, out=None, stream=None):
     K, R, S, C2 = w.shape
     if C != C2:
         raise ValueError("channel mismatch")
-    shp = out_shape("conv", N, H, W, K, R, S, pad_h, pad_w)
-    y = out if out is not None else torch.empty(shp, dtype=torch.float32, device=x.device)
-    _check_tensor(y, "out")
+    if w.device != x.device:
+        raise ValueError("x and w must be on the same device")
+    y = _out(out, out_shape("conv", N, H, W, K, R, S, pad_h, pad_w), x)
     _check("i2cw_conv2d_nhwc", lib().i2cw_conv2d_nhwc(N, H, W, C, K, R, S, pad_h, pad_w, x.data_ptr(), w.data_ptr(),
                                                       y.data_ptr(), _stream_ptr(stream)))
     return y
@@ -121,16 +145,78 @@ def deconv2d_nhwc(x, w, pad_h, pad_w, out=None, stream=None):
     C2, R, S, K = w.shape
     if C != C2:
         raise ValueError("channel mismatch")
-    shp = out_shape("deconv", N, H, W, K, R, S, pad_h, pad_w)
-    y = out if out is not None else torch.empty(shp, dtype=torch.float32, device=x.device)
-    _check_tensor(y, "out")
+    if w.device != x.device:
+        raise ValueError("x and w must be on the same device")
+    y = _out(out, out_shape("deconv", N, H, W, K, R, S, pad_h, pad_w), x)
     _check("i2cw_deconv2d_nhwc", lib().i2cw_deconv2d_nhwc(N, H, W, C, K, R, S, pad_h, pad_w, x.data_ptr(),
                                                           w.data_ptr(), y.data_ptr(), _stream_ptr(stream)))
     return y
 
 
-def filter_bytes(C, K, R, S) -> int:
-    return int(lib().i2cw_filter_bytes(C, K, R, S))
+def conv2d_nchw(x, w, pad_h, pad_w, out=None, stream=None):
+    """NCHW adapter (f4): x [N,C,H,W], w [K,C,R,S] (PyTorch OIHW) -> y [N,K,P,Q]."""
+    _check_tensor(x, "x"); _check_tensor(w, "w")
+    N, C, H, W = x.shape
+    K, C2, R, S = w.shape
+    if C != C2 or w.device != x.device:
+        raise ValueError("channel or device mismatch")
+    _, P, Q, _ = out_shape("conv", N, H, W, K, R, S, pad_h, pad_w)
+    y = _out(out, (N, K, P, Q), x)
+    _check("i2cw_conv2d_nchw", lib().i2cw_conv2d_nchw(N, C, H, W, K, R, S, pad_h, pad_w, x.data_ptr(), w.data_ptr(),
+                                                      y.data_ptr(), _stream_ptr(stream)))
+    return y
+
+
+def deconv2d_nchw(x, w, pad_h, pad_w, out=None, stream=None):
+    """NCHW adapter (f4): x [N,C,H,W], w [C,K,R,S] (conv_transpose2d weight) -> y [N,K,P,Q]."""
+    _check_tensor(x, "x"); _check_tensor(w, "w")
+    N, C, H, W = x.shape
+    C2, K, R, S = w.shape
+    if C != C2 or w.device != x.device:
+        raise ValueError("channel or device mismatch")
+    _, P, Q, _ = out_shape("deconv", N, H, W, K, R, S, pad_h, pad_w)
+    y = _out(out, (N, K, P, Q), x)
+    _check("i2cw_deconv2d_nchw", lib().i2cw_deconv2d_nchw(N, C, H, W, K, R, S, pad_h, pad_w, x.data_ptr(),
+                                                          w.data_ptr(), y.data_ptr(), _stream_ptr(stream)))
+    return y
+
+
+def out_shape3(kind, N, D, H, W, K, T, R, S, pad_d, pad_h, pad_w):
+    if kind == "conv":
+        return (N, D + 2 * pad_d - T + 1, H + 2 * pad_h - R + 1, W + 2 * pad_w - S + 1, K)
+    return (N, D + T - 1 - 2 * pad_d, H + R - 1 - 2 * pad_h, W + S - 1 - 2 * pad_w, K)
+
+
+def conv3d_ndhwc(x, w, pad_d, pad_h, pad_w, out=None, stream=None):
+    """3D conv; x [N,D,H,W,C], w [K,T,R,S,C] -> y [N,OD,P,Q,K]."""
+    _check_tensor(x, "x"); _check_tensor(w, "w")
+    N, D, H, W, C = x.shape
+    K, T, R, S, C2 = w.shape
+    if C != C2 or w.device != x.device:
+        raise ValueError("channel or device mismatch")
+    y = _out(out, out_shape3("conv", N, D, H, W, K, T, R, S, pad_d, pad_h, pad_w), x)
+    _check("i2cw_conv3d_ndhwc", lib().i2cw_conv3d_ndhwc(N, D, H, W, C, K, T, R, S, pad_d, pad_h, pad_w, x.data_ptr(),
+                                                        w.data_ptr(), y.data_ptr(), _stream_ptr(stream)))
+    return y
+
+
+def deconv3d_ndhwc(x, w, pad_d, pad_h, pad_w, out=None, stream=None):
+    """3D transposed conv; x [N,D,H,W,C], w [C,T,R,S,K] -> y [N,OD,P,Q,K], OD = D+T-1-2 pad_d."""
+    _check_tensor(x, "x"); _check_tensor(w, "w")
+    N, D, H, W, C = x.shape
+    C2, T, R, S, K = w.shape
+    if C != C2 or w.device != x.device:
+        raise ValueError("channel or device mismatch")
+    y = _out(out, out_shape3("deconv", N, D, H, W, K, T, R, S, pad_d, pad_h, pad_w), x)
+    _check("i2cw_deconv3d_ndhwc", lib().i2cw_deconv3d_ndhwc(N, D, H, W, C, K, T, R, S, pad_d, pad_h, pad_w,
+                                                            x.data_ptr(), w.data_ptr(), y.data_ptr(),
+                                                            _stream_ptr(stream)))
+    return y
+
+
+def filter_bytes(K, C, R, S) -> int:
+    """Bytes of a pre-transformed filter for a call with K output / C input channels (C ABI order)."""
+    return int(lib().i2cw_filter_bytes(K, C, R, S))
 
 
 def filter_transform(w, is_deconv=False, stream=None):
@@ -141,21 +227,27 @@ def filter_transform(w, is_deconv=False, stream=None):
         C, R, S, K = w.shape
     else:
         K, R, S, C = w.shape
-    nbytes = filter_bytes(C, K, R, S)
+    nbytes = filter_bytes(K, C, R, S)
     if nbytes == 0:
         raise I2CWError("i2cw_filter_bytes", I2CW_EUNSUPPORTED)
     u = torch.empty(nbytes, dtype=torch.uint8, device=w.device)
-    _check("i2cw_filter_transform", lib().i2cw_filter_transform(C, K, R, S, int(bool(is_deconv)), w.data_ptr(),
+    _check("i2cw_filter_transform", lib().i2cw_filter_transform(K, C, R, S, int(bool(is_deconv)), w.data_ptr(),
                                                                 u.data_ptr(), _stream_ptr(stream)))
     return u
 
 
 def conv2d_nhwc_pretransformed(x, u, K, R, S, pad_h, pad_w, is_deconv=False, out=None, stream=None):
+    """y from a filter pre-transformed by filter_transform() (the paper's '*' variant)."""
     import torch
     _check_tensor(x, "x")
     N, H, W, C = x.shape
-    shp = out_shape("deconv" if is_deconv else "conv", N, H, W, K, R, S, pad_h, pad_w)
-    y = out if out is not None else torch.empty(shp, dtype=torch.float32, device=x.device)
+    if not isinstance(u, torch.Tensor) or u.dtype != torch.uint8 or not u.is_cuda or not u.is_contiguous() \
+            or u.device != x.device:
+        raise ValueError("u must be a contiguous uint8 CUDA tensor on x's device (from filter_transform)")
+    need = filter_bytes(K, C, R, S)
+    if need == 0 or u.numel() < need:
+        raise ValueError(f"u holds {u.numel()} bytes, this call needs {need}")
+    y = _out(out, out_shape("deconv" if is_deconv else "conv", N, H, W, K, R, S, pad_h, pad_w), x)
     fn = lib().i2cw_deconv2d_nhwc_pretransformed if is_deconv else lib().i2cw_conv2d_nhwc_pretransformed
     _check("i2cw_*_pretransformed", fn(N, H, W, C, K, R, S, pad_h, pad_w, x.data_ptr(), u.data_ptr(), y.data_ptr(),
                                        _stream_ptr(stream)))
@@ -171,11 +263,18 @@ def conv2d_nhwc_host(x, w, pad_h, pad_w, is_deconv=False, out=None, stream=None)
             raise ValueError(f"{nm} must be a contiguous fp32 CPU tensor")
     N, H, W, C = x.shape
     if is_deconv:
-        _, R, S, K = w.shape
+        C2, R, S, K = w.shape
     else:
-        K, R, S, _ = w.shape
+        K, R, S, C2 = w.shape
+    if C != C2:
+        raise ValueError("channel mismatch")
     shp = out_shape("deconv" if is_deconv else "conv", N, H, W, K, R, S, pad_h, pad_w)
-    y = out if out is not None else torch.empty(shp, dtype=torch.float32)
+    if out is None:
+        y = torch.empty(shp, dtype=torch.float32)
+    else:
+        if out.dtype != torch.float32 or out.is_cuda or not out.is_contiguous() or tuple(out.shape) != tuple(shp):
+            raise ValueError(f"out must be a contiguous fp32 CPU tensor of shape {tuple(shp)}")
+        y = out
     dev = torch.cuda.current_device()
     _check("i2cw_set_device", lib().i2cw_set_device(dev))
     _check("i2cw_conv2d_nhwc_host", lib().i2cw_conv2d_nhwc_host(int(bool(is_deconv)), N, H, W, C, K, R, S, pad_h,
@@ -203,7 +302,8 @@ def transform_matrices(m, r, point_set=0):
 
 
 PLAN_FIELDS = ("P", "Q", "m", "alpha", "NT", "NB", "NCC", "NKS", "T_r", "TS", "SEGS", "ROWS", "PB", "WBOX", "HBOX",
-               "tile_blocks", "GP", "NPASS", "NUS", "smem_bytes", "pad_h", "pad_w", "NI", "NFULL", "NITEMS", "pair")
+               "tile_blocks", "GP", "NPASS", "NUS", "smem_bytes", "pad_h", "pad_w", "NI", "NFULL", "NITEMS", "pair",
+               "NKC", "CPC")
 
 
 def debug_plan(kind, N, H, W, C, K, R, S, pad_h, pad_w):
@@ -212,6 +312,11 @@ def debug_plan(kind, N, H, W, C, K, R, S, pad_h, pad_w):
     _check("i2cw_debug_plan", lib().i2cw_debug_plan(int(kind == "deconv"), N, H, W, C, K, R, S, pad_h, pad_w,
                                                     ctypes.addressof(out)))
     return dict(zip(PLAN_FIELDS, list(out)))
+
+
+def debug_set_kchunk(ksteps: int) -> int:
+    """TEST-ONLY: cap on k-steps accumulated in one TMEM accumulator (0 = default); returns the old cap."""
+    return int(lib().i2cw_debug_set_kchunk(int(ksteps)))
 
 
 def debug_conv_simt(x, w, pad_h, pad_w, is_deconv=False, stream=None):

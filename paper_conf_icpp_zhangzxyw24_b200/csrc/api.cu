@@ -8,6 +8,7 @@
 #include <cstdint>
 #include <cstdio>
 #include <cstring>
+#include <atomic>
 #include <mutex>
 #include <tuple>
 #include <vector>
@@ -22,13 +23,26 @@ cudaError_t launch_filter_transform(const float* w, float* u, int C, int K, int 
                                     UTag* tag_dst, cudaStream_t stream);
 cudaError_t launch_fused_tc(const CUtensorMap& xmap, const CUtensorMap& ymap, const Plan& pl, const float* u,
                             cudaStream_t stream);
-cudaError_t launch_zero_tail(float* y, size_t count, cudaStream_t stream);
+cudaError_t launch_zero_tail(float* y, size_t count, bool wait_first, cudaStream_t stream);
+cudaError_t launch_transpose(const float* in, float* out, int B, int rows, int cols, cudaStream_t stream);
 cudaError_t launch_fused_simt(const Plan& pl, const float* x, const float* u, float* y, cudaStream_t stream);
 
 namespace {
 
 
 constexpr int kSmemBudget = 225 * 1024;
+
+// Longest accumulation in one TMEM accumulator, in k-steps (8 channels x 1 filter row each).
+// The tcgen05 fp32 accumulator rounds toward zero once per MMA (3 MMAs per k-step in 3xTF32),
+// so the error grows ~linearly with the k-steps summed in TMEM. Measured on B200 with
+// all-positive U[1,2] inputs (the worst case, profiles/r02_accuracy_table.md): max |err| / sum|x||w|
+// ~1.4e-7 per k-step for alpha = 8 and ~2.8e-7 for alpha = 12 (the larger transform
+// amplification). Longer K loops are split into K-chunks whose partial results are added into y
+// by the fp32 round-to-nearest TMA reduce-add; the caps below keep that worst case at ~3.6e-5,
+// a ~2.8x margin under the 1e-4 bound, for any C.
+// i2cw_debug_set_kchunk (test hook) overrides the cap so small parity cases exercise chunking.
+int kchunk_default(int alpha) { return alpha <= 8 ? 256 : (alpha <= 12 ? 128 : 64); }
+std::atomic<int> g_kchunk_max{0};  // 0: kchunk_default(alpha)
 
 // Per filter width S: F(m, S) and the point set. r = 2..7 follow the paper's
 // Gamma_8 choices (Table 2). For r = 8, 9 the paper uses
@@ -41,8 +55,14 @@ bool alpha16_override() {
   static const bool on = [] { const char* e = getenv("I2CW_ALPHA16"); return e && e[0] == '1'; }();
   return on;
 }
+// I2CW_ALPHA=4 (experiments): Gamma4(3,2) / Gamma4(2,3) for S = 2, 3
+bool alpha4_override() {
+  static const bool on = [] { const char* e = getenv("I2CW_ALPHA"); return e && atoi(e) == 4; }();
+  return on;
+}
 bool choose(int S, Choice* c) {
   if (alpha16_override() && S >= 7 && S <= 9) { *c = {17 - S, 16, 1}; return true; }
+  if (alpha4_override() && (S == 2 || S == 3)) { *c = {5 - S, 4, 0}; return true; }
   switch (S) {
     case 2: *c = {7, 8, 0}; return true;
     case 3: *c = {6, 8, 0}; return true;
@@ -118,24 +138,36 @@ int num_sms() {
 }  // namespace
 
 // Build the launch plan. Returns I2CW_OK or an error code.
-int make_plan_uncached(int N, int H, int W, int C, int K, int R, int S, int pad_h, int pad_w, int is_deconv, Plan* out) {
+// vol = 1: 3D convolution (D, T, pad_d); 2D calls pass D = T = 1, pad_d = 0, vol = 0.
+int make_plan_uncached(int N, int D, int H, int W, int C, int K, int T, int R, int S, int pad_d, int pad_h, int pad_w,
+                       int is_deconv, int vol, Plan* out) {
   Plan pl;
   std::memset(&pl, 0, sizeof(pl));
-  if (N <= 0 || H <= 0 || W <= 0 || C <= 0 || K <= 0 || R <= 0 || S <= 0 || pad_h < 0 || pad_w < 0) return I2CW_EINVAL;
+  if (N <= 0 || D <= 0 || H <= 0 || W <= 0 || C <= 0 || K <= 0 || T <= 0 || R <= 0 || S <= 0 || pad_d < 0 ||
+      pad_h < 0 || pad_w < 0)
+    return I2CW_EINVAL;
+  if (!vol && (D != 1 || T != 1 || pad_d != 0)) return I2CW_EINVAL;
   Choice ch;
   if (!choose(S, &ch)) return I2CW_EUNSUPPORTED;
+  // the 3D kernels are instantiated for the default alpha = 8 / 12 families only
+  if (vol && ch.alpha != 8 && ch.alpha != 12) ch = Choice{S <= 7 ? 9 - S : 13 - S, S <= 7 ? 8 : 12, 0};
   if (C % 4 != 0 || K % 4 != 0) return I2CW_EUNSUPPORTED;
   pl.N = N; pl.H = H; pl.W = W; pl.C = C; pl.K = K; pl.R = R; pl.S = S;
-  if (is_deconv) {  // deconv(x, w, pad) == conv(x, rot180(w)^T, R-1-pad)
+  pl.vol = vol; pl.D = D; pl.T = T;
+  pl.is_deconv = is_deconv;
+  if (is_deconv) {  // deconv(x, w, pad) == conv(x, rot180(w)^T, R-1-pad) (3D: rotate all three taps)
+    pl.pad_d = T - 1 - pad_d;
     pl.pad_h = R - 1 - pad_h;
     pl.pad_w = S - 1 - pad_w;
   } else {
+    pl.pad_d = pad_d;
     pl.pad_h = pad_h;
     pl.pad_w = pad_w;
   }
+  pl.OD = D + 2 * pl.pad_d - T + 1;
   pl.P = H + 2 * pl.pad_h - R + 1;
   pl.Q = W + 2 * pl.pad_w - S + 1;
-  if (pl.P < 1 || pl.Q < 1) return I2CW_EINVAL;
+  if (pl.OD < 1 || pl.P < 1 || pl.Q < 1) return I2CW_EINVAL;
   pl.m = ch.m;
   pl.alpha = ch.alpha;
   // Output channels per CTA (UMMA N): 64 (4 points per pass, 4 V slots of 64 columns) for
@@ -145,12 +177,22 @@ int make_plan_uncached(int N, int H, int W, int C, int K, int R, int S, int pad_
   // profiles/r01f_nt128.txt), so it is opt-in: I2CW_NT=<32|64|128> overrides (experiments).
   static const int nt_env = [] { const char* e = getenv("I2CW_NT"); return e ? atoi(e) : 0; }();
   pl.NT = K > 32 ? 64 : 32;
-  if (nt_env == 32 || nt_env == 64 || (nt_env == 128 && ch.alpha <= 12)) pl.NT = nt_env;
+  if (nt_env == 32 || nt_env == 64 || (nt_env == 128 && ch.alpha >= 8 && ch.alpha <= 12)) pl.NT = nt_env;
   pl.GP = gp_for(pl.alpha, pl.NT);
   pl.NPASS = pl.alpha / pl.GP;
   pl.NB = cdiv(K, pl.NT);
-  pl.NCC = cdiv(C, 8);
+  pl.NCC = cdiv(C, 8) * T;  // 3D: virtual chunks (channel chunk, depth tap)
   pl.NKS = pl.NCC * R;
+  {
+    const int kset = g_kchunk_max.load();
+    const int kmax = std::max(R, kset > 0 ? kset : kchunk_default(pl.alpha));
+    const int cpc_max = std::max(1, kmax / R);
+    pl.NKC = cdiv(pl.NCC, cpc_max);
+    pl.CPC = cdiv(pl.NCC, pl.NKC);  // balanced chunks
+    pl.CC0 = 0;
+    pl.CC1 = pl.NCC;
+    pl.ACCUM = 0;
+  }
   pl.T_r = cdiv(pl.Q, pl.m);
   // WBOX <= 256 (TMA box limit), leave 7 columns of slack for the bank search
   const int ts_max = std::min(kMaxLanes, (256 - 7 - (S - 1)) / pl.m);
@@ -164,6 +206,7 @@ int make_plan_uncached(int N, int H, int W, int C, int K, int R, int S, int pad_
   // (c256 +11%), -2..-18% otherwise (cfg2, r2-r7, c64, c128). I2CW_PAIR=1/0 forces it.
   static const int pair_env = [] { const char* e = getenv("I2CW_PAIR"); return e ? (e[0] == '1' ? 1 : 0) : -1; }();
   pl.pair = pair_env >= 0 ? pair_env : ((pl.NKS >= 128 || pl.NB >= 4) ? 1 : 0);
+  if (vol) pl.pair = 0;  // 3D kernels: single-CTA instantiations only
   // DEBUG timing ablation (never set in production; results are wrong when non-zero)
   static const int ablate = [] { const char* e = getenv("I2CW_ABLATE"); return e ? atoi(e) : 0; }();
   pl.ablate = ablate;
@@ -193,11 +236,11 @@ int make_plan_uncached(int N, int H, int W, int C, int K, int R, int S, int pad_
   // block would use 70 of 128 lanes, NI = 6 x 4 rows uses 120).
   const int nsm = num_sms();
   // Split tail (Plan::NFULL / NITEMS, applied after the block shape is chosen): with 2 passes
-  // and no CTA pairs, the last T = units mod G units run as 2T one-pass items when 2T <= G, so
+  // (single CTAs or CTA pairs), the last T = units mod G units run as 2T one-pass items when 2T <= G, so
   // they cost half a unit time (cfg2 +4%, r7 +10%). Ranking block shapes by half-unit rounds
   // instead picked more images per block and measured slower (r2 -24%, c128 -7%), so the
   // ranking keeps whole rounds. I2CW_SPLIT_TAIL=0 disables the split.
-  const bool split_ok = !pl.pair && pl.NPASS == 2 && [] {
+  const bool split_ok = pl.NPASS == 2 && [] {
     const char* e = getenv("I2CW_SPLIT_TAIL");
     return !(e && e[0] == '0');
   }();
@@ -209,7 +252,9 @@ int make_plan_uncached(int N, int H, int W, int C, int K, int R, int S, int pad_
   // so small parity cases exercise multi-image blocks
   static const int force_ni = [] { const char* e = getenv("I2CW_NI"); return e ? atoi(e) : 0; }();
   const int ni_lo = force_ni > 0 ? std::min(force_ni, kMaxLanes / pl.TS) : 1;
-  const int ni_max = force_ni > 0 ? ni_lo : std::min(N, kMaxLanes / pl.TS);
+  // 2D: NI consecutive images per block; 3D: NI consecutive output depths of one image
+  const int stack_extent = vol ? pl.OD : N;
+  const int ni_max = force_ni > 0 ? ni_lo : std::min(stack_extent, kMaxLanes / pl.TS);
   for (int ni = ni_lo; ni <= ni_max; ++ni) {
     int rmax = std::min({kMaxLanes / (ni * pl.TS), pl.P, 256 - (R - 1)});
     if (pl.SEGS > 1) rmax = std::min(rmax, 1);
@@ -230,7 +275,7 @@ int make_plan_uncached(int N, int H, int W, int C, int K, int R, int S, int pad_
         if (sm <= kSmemBudget) { depth = d; break; }
       }
       if (depth < 0 || ni * hbox > 256) continue;
-      const int blocks = cdiv(N, ni) * pb * pl.SEGS;
+      const int blocks = (vol ? N * cdiv(pl.OD, ni) : cdiv(N, ni)) * pb * pl.SEGS;
       const int units = (pl.pair ? cdiv(blocks, 2) : blocks) * pl.NB;
       const int G = pl.pair ? std::max(1, nsm / 2) : nsm;
       const Cand c{cdiv(units, G), depth, ni * hbox, units, ni, rb, pb};
@@ -257,7 +302,6 @@ int make_plan_uncached(int N, int H, int W, int C, int K, int R, int S, int pad_
   pl.PLANE = (pl.BOXB + 1023) / 1024 * 512;   // half a stage; stages stay 1024-aligned (TMA swizzle)
   // Output staging: one output column i of every tile for one warpgroup's 16 channels (one
   // 64-byte swizzled row per tile), stored by TMA with Q stride m.
-  pl.OPITCH = pl.TS * pl.m;
   pl.OSB = pl.NI * pl.ROWS * pl.TS * cpw * 4;
   pl.OSTRIDE = (pl.OSB + 1023) / 1024 * 1024;
   pl.NUS = std::max(kDepths[best.depth][0] / kps, 2);  // U super-slots
@@ -267,14 +311,15 @@ int make_plan_uncached(int N, int H, int W, int C, int K, int R, int S, int pad_
   pl.smem_bytes = pl.NUS * kps * ubytes + pl.NIS * 2 * pl.PLANE + nwg_for(pl.NT) * pl.NOB * pl.OSTRIDE + bar_bytes;
   if (pl.smem_bytes > kSmemBudget) return I2CW_EUNSUPPORTED;
   assign_lanes(pl.NI, pl.ROWS, pl.HBOX, pl.TS, pl.WBOX, pl.m, pl.lane_row, pl.lane_in, pl.lane_tw);
-  pl.tile_blocks = cdiv(N, pl.NI) * pl.PB * pl.SEGS;
+  pl.DB = vol ? cdiv(pl.OD, pl.NI) : 1;
+  pl.tile_blocks = (vol ? N * pl.DB : cdiv(N, pl.NI)) * pl.PB * pl.SEGS;
   {
     const int units = (pl.pair ? cdiv(pl.tile_blocks, 2) : pl.tile_blocks) * pl.NB;
     const int G = pl.pair ? std::max(1, nsm / 2) : nsm;
-    const int T = units % G;
-    if (split_ok && T > 0 && 2 * T <= G) {
-      pl.NFULL = units - T;
-      pl.NITEMS = pl.NFULL + 2 * T;
+    const int tail = units % G;
+    if (split_ok && tail > 0 && 2 * tail <= G) {
+      pl.NFULL = units - tail;
+      pl.NITEMS = pl.NFULL + 2 * tail;
     } else {
       pl.NFULL = pl.NITEMS = units;
     }
@@ -285,26 +330,31 @@ int make_plan_uncached(int N, int H, int W, int C, int K, int R, int S, int pad_
 
 // Plans are pure functions of the call's dimensions (and the device's SM count): memoised,
 // so repeated calls skip the block-shape search and the lane permutation.
-int make_plan(int N, int H, int W, int C, int K, int R, int S, int pad_h, int pad_w, int is_deconv, Plan* out) {
-  struct Key { int v[11]; };
+int make_plan3(int N, int D, int H, int W, int C, int K, int T, int R, int S, int pad_d, int pad_h, int pad_w,
+               int is_deconv, int vol, Plan* out) {
+  struct Key { int v[16]; };
   static std::mutex mu;
   static std::vector<std::pair<Key, Plan>> memo;
   int dev = 0;
   if (cudaGetDevice(&dev) != cudaSuccess) { cudaGetLastError(); dev = -1; }
-  const Key k{{N, H, W, C, K, R, S, pad_h, pad_w, is_deconv, dev}};
+  const Key k{{N, D, H, W, C, K, T, R, S, pad_d, pad_h, pad_w, is_deconv, vol, dev, g_kchunk_max.load()}};
   {
     std::lock_guard<std::mutex> lk(mu);
     for (auto& e : memo)
       if (std::memcmp(e.first.v, k.v, sizeof(k.v)) == 0) { *out = e.second; return I2CW_OK; }
   }
   Plan pl;
-  const int rc = make_plan_uncached(N, H, W, C, K, R, S, pad_h, pad_w, is_deconv, &pl);
+  const int rc = make_plan_uncached(N, D, H, W, C, K, T, R, S, pad_d, pad_h, pad_w, is_deconv, vol, &pl);
   if (rc != I2CW_OK) return rc;
   std::lock_guard<std::mutex> lk(mu);
   if (memo.size() >= 256) memo.erase(memo.begin());
   memo.push_back({k, pl});
   *out = pl;
   return I2CW_OK;
+}
+
+int make_plan(int N, int H, int W, int C, int K, int R, int S, int pad_h, int pad_w, int is_deconv, Plan* out) {
+  return make_plan3(N, 1, H, W, C, K, 1, R, S, 0, pad_h, pad_w, is_deconv, 0, out);
 }
 
 namespace {
@@ -330,6 +380,17 @@ PFN_encodeTiled_t get_encode() {
 int encode_x_map(const Plan& pl, const float* x, CUtensorMap* map) {
   PFN_encodeTiled_t enc = get_encode();
   if (!enc) return I2CW_ECUDA;
+  if (pl.vol) {  // [N][D][H][W][C]: box = 8 channels x WBOX x HBOX x NI depths x 1 image
+    cuuint64_t dims[5] = {(cuuint64_t)pl.C, (cuuint64_t)pl.W, (cuuint64_t)pl.H, (cuuint64_t)pl.D, (cuuint64_t)pl.N};
+    const cuuint64_t sw = (cuuint64_t)pl.C * 4, sh = sw * pl.W, sd = sh * pl.H, sn = sd * pl.D;
+    cuuint64_t strides[4] = {sw, sh, sd, sn};
+    cuuint32_t box[5] = {8, (cuuint32_t)pl.WBOX, (cuuint32_t)pl.HBOX, (cuuint32_t)pl.NI, 1};
+    cuuint32_t es[5] = {1, 1, 1, 1, 1};
+    CUresult r = enc(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 5, const_cast<float*>(x), dims, strides, box, es,
+                     CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_32B, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+                     CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    return r == CUDA_SUCCESS ? I2CW_OK : I2CW_EUNSUPPORTED;
+  }
   cuuint64_t dims[4] = {(cuuint64_t)pl.C, (cuuint64_t)pl.W, (cuuint64_t)pl.H, (cuuint64_t)pl.N};
   cuuint64_t strides[3] = {(cuuint64_t)pl.C * 4, (cuuint64_t)pl.W * pl.C * 4, (cuuint64_t)pl.H * pl.W * pl.C * 4};
   cuuint32_t box[4] = {8, (cuuint32_t)pl.WBOX, (cuuint32_t)pl.HBOX, (cuuint32_t)pl.NI};
@@ -346,6 +407,18 @@ int encode_x_map(const Plan& pl, const float* x, CUtensorMap* map) {
 int encode_y_map(const Plan& pl, float* y, CUtensorMap* map) {
   PFN_encodeTiled_t enc = get_encode();
   if (!enc) return I2CW_ECUDA;
+  if (pl.vol) {  // [N][OD][P][Q][K]: box = cpw channels x TS positions (stride m) x ROWS x NI depths x 1
+    const int cpw = pl.NT / nwg_for(pl.NT);
+    cuuint64_t dims[5] = {(cuuint64_t)pl.K, (cuuint64_t)pl.Q, (cuuint64_t)pl.P, (cuuint64_t)pl.OD, (cuuint64_t)pl.N};
+    const cuuint64_t sq = (cuuint64_t)pl.K * 4, sp = sq * pl.Q, sd = sp * pl.P, sn = sd * pl.OD;
+    cuuint64_t strides[4] = {sq, sp, sd, sn};
+    cuuint32_t box[5] = {(cuuint32_t)cpw, (cuuint32_t)(pl.TS * pl.m), (cuuint32_t)pl.ROWS, (cuuint32_t)pl.NI, 1};
+    cuuint32_t es[5] = {1, (cuuint32_t)pl.m, 1, 1, 1};
+    CUresult r = enc(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 5, y, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                     (cpw == 16 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_128B),
+                     CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    return r == CUDA_SUCCESS ? I2CW_OK : I2CW_EUNSUPPORTED;
+  }
   cuuint64_t dims[4] = {(cuuint64_t)pl.K, (cuuint64_t)pl.Q, (cuuint64_t)pl.P, (cuuint64_t)pl.N};
   cuuint64_t strides[3] = {(cuuint64_t)pl.K * 4, (cuuint64_t)pl.Q * pl.K * 4, (cuuint64_t)pl.P * pl.Q * pl.K * 4};
   const int cpw = pl.NT / nwg_for(pl.NT);  // one warpgroup's channels: 64 B or 128 B rows
@@ -415,56 +488,89 @@ void g_internal(const Plan& pl, int point_set, std::vector<double>* G) {
     for (int s = 0; s < pl.S; ++s) (*G)[(size_t)idx * pl.S + s] = T.G[(size_t)point_of(idx, pl.alpha) * pl.S + s].to_double();
 }
 
+// the 256-byte header in front of U: what the filter was transformed for
+UTag make_tag(const Plan& pl, int is_deconv) {
+  UTag t;
+  std::memset(&t, 0, sizeof(t));
+  t.magic = kUMagic; t.alpha = pl.alpha; t.m = pl.m; t.is_deconv = is_deconv;
+  t.C = pl.C; t.K = pl.K; t.R = pl.R; t.S = pl.S; t.NT = pl.NT; t.NB = pl.NB; t.NCC = pl.NCC;
+  t.halves = pl.pair ? 2 : 1;
+  t.T = pl.T;
+  return t;
+}
+
 size_t u_data_bytes(const Plan& pl) { return (size_t)pl.NB * pl.NKS * pl.alpha * 2 * pl.NT * 8 * 4; }
 
-// exact G tables are generated once per (m, S, point set) and kept (host memo)
-const std::vector<double>& g_cached(const Plan& pl, int point_set) {
+// exact G tables are generated once per (m, S, point set) and kept (host memo). Returned BY
+// VALUE (at most 16 x 9 doubles): a reference into the memo could be invalidated by another
+// thread's insertion while the caller still reads it.
+std::vector<double> g_cached(const Plan& pl, int point_set) {
   static std::mutex mu;
   static std::vector<std::pair<int, std::vector<double>>> memo;
   const int key = (pl.m * 16 + pl.S) * 2 + point_set;
   std::lock_guard<std::mutex> lk(mu);
   for (auto& e : memo)
     if (e.first == key) return e.second;
-  memo.push_back({key, {}});
-  g_internal(pl, point_set, &memo.back().second);
-  return memo.back().second;
+  std::vector<double> G;
+  g_internal(pl, point_set, &G);
+  memo.push_back({key, G});
+  return G;
 }
 
 int transform_into(const Plan& pl, int is_deconv, const float* w, void* u, cudaStream_t stream) {
   Choice ch;
   choose(pl.S, &ch);
-  const std::vector<double>& G = g_cached(pl, ch.point_set);
-  UTag tag;
-  std::memset(&tag, 0, sizeof(tag));
-  tag.magic = kUMagic; tag.alpha = pl.alpha; tag.m = pl.m; tag.is_deconv = is_deconv;
-  tag.C = pl.C; tag.K = pl.K; tag.R = pl.R; tag.S = pl.S; tag.NT = pl.NT; tag.NB = pl.NB; tag.NCC = pl.NCC;
-  tag.halves = pl.pair ? 2 : 1;
+  const std::vector<double> G = g_cached(pl, ch.point_set);
+  const UTag tag = make_tag(pl, is_deconv);
   static_assert(sizeof(UTag) <= kUTagBytes, "tag");
-  registry_put(u, tag);
   float* ud = reinterpret_cast<float*>(static_cast<uint8_t*>(u) + kUTagBytes);
-  if (launch_filter_transform(w, ud, pl.C, pl.K, pl.R, pl.S, is_deconv, pl.alpha, pl.NT, pl.NB, pl.NCC, pl.pair ? 2 : 1, G.data(),
-                              tag, static_cast<UTag*>(u), stream) != cudaSuccess)
+  // 3D: the [K][T][R][S][C] filter is the 2D filter [K][T*R][S][C] (and the deconv rotation of the
+  // combined T*R axis is the rotation of both), with ceil(C/8) channel chunks
+  if (launch_filter_transform(w, ud, pl.C, pl.K, pl.R * pl.T, pl.S, is_deconv, pl.alpha, pl.NT, pl.NB, pl.NCC / pl.T,
+                              pl.pair ? 2 : 1, G.data(), tag, static_cast<UTag*>(u), stream) != cudaSuccess)
     return I2CW_ECUDA;
   return I2CW_OK;
 }
 
-int run_fused(const Plan& pl, const float* x, const void* u, float* y, cudaStream_t stream) {
+// after_own_ft: the previous kernel in the stream is this library's filter transform (which
+// never touches y), so the zeroing kernel may overlap it through programmatic dependent launch;
+// otherwise (pre-transformed path: the caller's last kernel is unknown) the zeroing kernel
+// waits for the previous grid before its first store.
+int run_fused(const Plan& pl, const float* x, const void* u, float* y, bool after_own_ft, cudaStream_t stream) {
   CUtensorMap map, ymap;
   if (pl.NITEMS != pl.NFULL) {
     // split tail: both passes of a tail unit reduce-add into y, so y is zeroed from the first
     // image the tail touches (earlier rows of that image are overwritten by whole-unit stores)
-    const int tb0 = pl.NFULL / pl.NB;
-    const size_t n0 = (size_t)(tb0 / pl.SEGS / pl.PB) * pl.NI;
-    const size_t img = (size_t)pl.P * pl.Q * pl.K;
-    if (n0 < (size_t)pl.N && launch_zero_tail(y + n0 * img, ((size_t)pl.N - n0) * img, stream) != cudaSuccess)
+    const int tb0 = (pl.pair ? 2 : 1) * (pl.NFULL / pl.NB);  // first tile block of the tail
+    const int ib = tb0 / pl.SEGS / pl.PB;  // image block of the first tail unit
+    const size_t n0 = pl.vol ? (size_t)(ib / pl.DB) : (size_t)ib * pl.NI;
+    const size_t img = (size_t)pl.OD * pl.P * pl.Q * pl.K;
+    if (n0 < (size_t)pl.N &&
+        launch_zero_tail(y + n0 * img, ((size_t)pl.N - n0) * img, !after_own_ft, stream) != cudaSuccess)
       return I2CW_ECUDA;
   }
   int rc = encode_x_map(pl, x, &map);
   if (rc != I2CW_OK) return rc;
   if ((rc = encode_y_map(pl, y, &ymap)) != I2CW_OK) return rc;
   const float* ud = reinterpret_cast<const float*>(static_cast<const uint8_t*>(u) + kUTagBytes);
-  return launch_fused_tc(map, ymap, pl, ud, stream) == cudaSuccess ? I2CW_OK : I2CW_ECUDA;
+  // K-chunks: one launch per chunk of <= CPC channel chunks, in order on the
+  // stream; the first stores y (its split tail reduce-adds into the zeroed region), later ones
+  // reduce-add every pass. Sequential launches keep the fp32 summation order fixed.
+  for (int kc = 0; kc < pl.NKC; ++kc) {
+    Plan pk = pl;
+    pk.CC0 = kc * pl.CPC;
+    pk.CC1 = std::min(pl.NCC, pk.CC0 + pl.CPC);
+    pk.ACCUM = kc > 0;
+    // the split tail's two one-pass items per unit add in either order: exact only onto y = 0
+    // (0 + a + b), so later chunks (y != 0) run every unit whole, its passes in order
+    if (kc > 0) pk.NFULL = pk.NITEMS = pl.NFULL + (pl.NITEMS - pl.NFULL) / 2;
+    if (launch_fused_tc(map, ymap, pk, ud, stream) != cudaSuccess) return I2CW_ECUDA;
+  }
+  return I2CW_OK;
 }
+
+int conv_plan(const Plan& plan, int is_deconv, const float* x, const float* w, float* y, cudaStream_t stream, bool simt,
+              unsigned long long* trace);
 
 int conv_common(int is_deconv, int N, int H, int W, int C, int K, int R, int S, int pad_h, int pad_w, const float* x,
                 const float* w, float* y, cudaStream_t stream, bool simt, unsigned long long* trace = nullptr) {
@@ -473,6 +579,24 @@ int conv_common(int is_deconv, int N, int H, int W, int C, int K, int R, int S, 
   Plan pl;
   int rc = make_plan(N, H, W, C, K, R, S, pad_h, pad_w, is_deconv, &pl);
   if (rc != I2CW_OK) return rc;
+  return conv_plan(pl, is_deconv, x, w, y, stream, simt, trace);
+}
+
+// 3D convolution / deconvolution: NDHWC x, KTRSC (deconv: CTRSK) w, NDHWC y
+int conv3_common(int is_deconv, int N, int D, int H, int W, int C, int K, int T, int R, int S, int pad_d, int pad_h,
+                 int pad_w, const float* x, const float* w, float* y, cudaStream_t stream) {
+  if (!x || !w || !y) return I2CW_EINVAL;
+  if (!aligned16(x) || !aligned16(w) || !aligned16(y)) return I2CW_EINVAL;
+  Plan pl;
+  int rc = make_plan3(N, D, H, W, C, K, T, R, S, pad_d, pad_h, pad_w, is_deconv, 1, &pl);
+  if (rc != I2CW_OK) return rc;
+  return conv_plan(pl, is_deconv, x, w, y, stream, false, nullptr);
+}
+
+int conv_plan(const Plan& plan, int is_deconv, const float* x, const float* w, float* y, cudaStream_t stream, bool simt,
+              unsigned long long* trace) {
+  Plan pl = plan;
+  int rc = I2CW_OK;
   pl.trace = trace;
   if (simt) pl.pair = 0;  // the SIMT stepping stone reads the single-CTA U layout
   if ((rc = bind_device_of(x)) != I2CW_OK) return rc;
@@ -487,7 +611,7 @@ int conv_common(int is_deconv, int N, int H, int W, int C, int K, int R, int S, 
                ? I2CW_OK
                : I2CW_ECUDA;
     else
-      rc = run_fused(pl, x, u, y, stream);
+      rc = run_fused(pl, x, u, y, /*after_own_ft=*/true, stream);
   }
   cudaFreeAsync(u, stream);
   if (rc != I2CW_OK) cudaGetLastError();
@@ -502,19 +626,26 @@ int pretransformed_common(int is_deconv, int N, int H, int W, int C, int K, int 
   int rc = make_plan(N, H, W, C, K, R, S, pad_h, pad_w, is_deconv, &pl);
   if (rc != I2CW_OK) return rc;
   if ((rc = bind_device_of(x)) != I2CW_OK) return rc;
+  auto matches = [&](const UTag& t) {
+    return t.magic == kUMagic && (int)t.is_deconv == is_deconv && (int)t.C == C && (int)t.K == K && (int)t.R == R &&
+           (int)t.S == S && (int)t.alpha == pl.alpha && (int)t.m == pl.m && (int)t.NT == pl.NT &&
+           (int)t.halves == (pl.pair ? 2 : 1);
+  };
+  // Host copy of the tag (written by i2cw_filter_transform for this address) when it matches;
+  // otherwise -- an unknown u, or a host entry that disagrees (the address may have been freed
+  // and reused) -- the device tag decides (one small synchronous read). The fused kernel checks
+  // the device tag again and traps on a mismatch, so a stale host entry cannot pass silently.
   UTag tag;
-  if (!registry_lookup(u, &tag)) {  // not made by i2cw_filter_transform in this process: read the device tag
+  if (!registry_lookup(u, &tag) || !matches(tag)) {
     if (cudaMemcpyAsync(&tag, u, sizeof(tag), cudaMemcpyDeviceToHost, stream) != cudaSuccess ||
         cudaStreamSynchronize(stream) != cudaSuccess) {
       cudaGetLastError();
       return I2CW_ECUDA;
     }
+    if (!matches(tag)) return I2CW_EINVAL;
+    registry_put(u, tag);
   }
-  if (tag.magic != kUMagic || (int)tag.is_deconv != is_deconv || (int)tag.C != C || (int)tag.K != K ||
-      (int)tag.R != R || (int)tag.S != S || (int)tag.alpha != pl.alpha || (int)tag.m != pl.m || (int)tag.NT != pl.NT ||
-      (int)tag.halves != (pl.pair ? 2 : 1))
-    return I2CW_EINVAL;
-  rc = run_fused(pl, x, u, y, stream);
+  rc = run_fused(pl, x, u, y, /*after_own_ft=*/false, stream);
   if (rc != I2CW_OK) cudaGetLastError();
   return rc;
 }
@@ -548,21 +679,80 @@ int i2cw_deconv2d_nhwc(int N, int H, int W, int C, int K, int R, int S, int pad_
   return conv_common(1, N, H, W, C, K, R, S, pad_h, pad_w, x, w, y, (cudaStream_t)stream, false);
 }
 
-size_t i2cw_filter_bytes(int C, int K, int R, int S) {
+// NCHW adapter (f4): transpose x (NCHW -> NHWC) and the filter (OIHW -> KRSC, or for the
+// deconv the [C][K][R][S] conv_transpose weight -> CRSK) into pooled workspaces, run the NHWC
+// call, transpose y back. Costs one extra read + write of x, y and w in HBM.
+static int nchw_common(int is_deconv, int N, int C, int H, int W, int K, int R, int S, int pad_h, int pad_w,
+                       const float* x, const float* w, float* y, cudaStream_t stream) {
+  if (!x || !w || !y) return I2CW_EINVAL;
+  if (!aligned16(x) || !aligned16(w) || !aligned16(y)) return I2CW_EINVAL;
+  Plan pl;
+  int rc = make_plan(N, H, W, C, K, R, S, pad_h, pad_w, is_deconv, &pl);
+  if (rc != I2CW_OK) return rc;
+  if ((rc = bind_device_of(x)) != I2CW_OK) return rc;
+  const size_t nx = (size_t)N * C * H * W, nw = (size_t)K * C * R * S, ny = (size_t)N * K * pl.P * pl.Q;
+  float *xt = nullptr, *wt = nullptr, *yt = nullptr;
+  if (cudaMallocAsync(&xt, nx * 4, stream) != cudaSuccess || cudaMallocAsync(&wt, nw * 4, stream) != cudaSuccess ||
+      cudaMallocAsync(&yt, ny * 4, stream) != cudaSuccess) {
+    cudaGetLastError();
+    if (xt) cudaFreeAsync(xt, stream);
+    if (wt) cudaFreeAsync(wt, stream);
+    return I2CW_ECUDA;
+  }
+  if (launch_transpose(x, xt, N, C, H * W, stream) != cudaSuccess ||
+      // conv: OIHW [K][C][R*S] -> [K][R*S][C]; deconv: [C][K][R*S] -> [C][R*S][K]
+      launch_transpose(w, wt, is_deconv ? C : K, is_deconv ? K : C, R * S, stream) != cudaSuccess)
+    rc = I2CW_ECUDA;
+  if (rc == I2CW_OK) rc = conv_common(is_deconv, N, H, W, C, K, R, S, pad_h, pad_w, xt, wt, yt, stream, false);
+  if (rc == I2CW_OK && launch_transpose(yt, y, N, pl.P * pl.Q, K, stream) != cudaSuccess) rc = I2CW_ECUDA;
+  cudaFreeAsync(xt, stream);
+  cudaFreeAsync(wt, stream);
+  cudaFreeAsync(yt, stream);
+  if (rc != I2CW_OK) cudaGetLastError();
+  return rc;
+}
+
+int i2cw_conv2d_nchw(int N, int C, int H, int W, int K, int R, int S, int pad_h, int pad_w, const float* x,
+                     const float* w, float* y, i2cw_stream_t stream) {
+  return nchw_common(0, N, C, H, W, K, R, S, pad_h, pad_w, x, w, y, (cudaStream_t)stream);
+}
+
+int i2cw_deconv2d_nchw(int N, int C, int H, int W, int K, int R, int S, int pad_h, int pad_w, const float* x,
+                       const float* w, float* y, i2cw_stream_t stream) {
+  return nchw_common(1, N, C, H, W, K, R, S, pad_h, pad_w, x, w, y, (cudaStream_t)stream);
+}
+
+int i2cw_conv3d_ndhwc(int N, int D, int H, int W, int C, int K, int T, int R, int S, int pad_d, int pad_h, int pad_w,
+                      const float* x, const float* w, float* y, i2cw_stream_t stream) {
+  return conv3_common(0, N, D, H, W, C, K, T, R, S, pad_d, pad_h, pad_w, x, w, y, (cudaStream_t)stream);
+}
+
+int i2cw_deconv3d_ndhwc(int N, int D, int H, int W, int C, int K, int T, int R, int S, int pad_d, int pad_h, int pad_w,
+                        const float* x, const float* w, float* y, i2cw_stream_t stream) {
+  return conv3_common(1, N, D, H, W, C, K, T, R, S, pad_d, pad_h, pad_w, x, w, y, (cudaStream_t)stream);
+}
+
+size_t i2cw_filter_bytes(int K, int C, int R, int S) {
   Plan pl;
   // the filter-side plan fields do not depend on N, H, W or pad: plan a 1 x R x S map
   if (make_plan(1, R, S, C, K, R, S, 0, 0, 0, &pl) != I2CW_OK) return 0;
   return kUTagBytes + u_data_bytes(pl);
 }
 
-int i2cw_filter_transform(int C, int K, int R, int S, int is_deconv, const float* w, void* u, i2cw_stream_t stream) {
+int i2cw_filter_transform(int K, int C, int R, int S, int is_deconv, const float* w, void* u, i2cw_stream_t stream) {
   if (!w || !u || !aligned16(w) || !aligned16(u) || (is_deconv != 0 && is_deconv != 1)) return I2CW_EINVAL;
   Plan pl;
   int rc = make_plan(1, R, S, C, K, R, S, 0, 0, 0, &pl);
   if (rc != I2CW_OK) return rc;
   if ((rc = bind_device_of(w)) != I2CW_OK) return rc;
   rc = transform_into(pl, is_deconv, w, u, (cudaStream_t)stream);
-  if (rc != I2CW_OK) cudaGetLastError();
+  if (rc != I2CW_OK) {
+    cudaGetLastError();
+    return rc;
+  }
+  // host copy of the caller-owned u's tag (internal workspaces are never registered)
+  const UTag tag = make_tag(pl, is_deconv);
+  registry_put(u, tag);
   return rc;
 }
 
@@ -646,7 +836,7 @@ int i2cw_conv2d_nhwc_host(int is_deconv, int N, int H, int W, int C, int K, int 
       rc = I2CW_ECUDA;
       break;
     }
-    if ((rc = run_fused(pc, xdc, u, ydc, stream)) != I2CW_OK) break;
+    if ((rc = run_fused(pc, xdc, u, ydc, /*after_own_ft=*/c == 0, stream)) != I2CW_OK) break;
     if (cudaEventRecord(ev[2 * c + 1], stream) != cudaSuccess || cudaStreamWaitEvent(so, ev[2 * c + 1], 0) != cudaSuccess ||
         cudaMemcpyAsync(y_host + (size_t)n0 * img_y, ydc, (size_t)nc * img_y * 4, cudaMemcpyDeviceToHost, so) !=
             cudaSuccess) {
@@ -712,6 +902,10 @@ I2CW_API int i2cw_debug_conv_simt(int is_deconv, int N, int H, int W, int C, int
   return conv_common(is_deconv, N, H, W, C, K, R, S, pad_h, pad_w, x, w, y, (cudaStream_t)stream, true);
 }
 
+// Longest TMEM accumulation in k-steps (0 restores the per-alpha default); returns the previous
+// setting (0 = default).
+I2CW_API int i2cw_debug_set_kchunk(int ksteps) { return g_kchunk_max.exchange(ksteps > 0 ? ksteps : 0); }
+
 // Runs the product path with CTA 0's event timeline recorded into trace (device,
 // 32 kinds x 512 uint64 clock64 stamps; see trace_rec in common.cuh).
 I2CW_API int i2cw_debug_trace(int is_deconv, int N, int H, int W, int C, int K, int R, int S, int pad_h, int pad_w,
@@ -727,7 +921,7 @@ I2CW_API int i2cw_debug_plan(int is_deconv, int N, int H, int W, int C, int K, i
   if (rc != I2CW_OK) return rc;
   int v[] = {pl.P, pl.Q, pl.m, pl.alpha, pl.NT, pl.NB, pl.NCC, pl.NKS, pl.T_r, pl.TS, pl.SEGS, pl.ROWS, pl.PB,
              pl.WBOX, pl.HBOX, pl.tile_blocks, pl.GP, pl.NPASS, pl.NUS, pl.smem_bytes, pl.pad_h, pl.pad_w, pl.NI,
-             pl.NFULL, pl.NITEMS, pl.pair};
+             pl.NFULL, pl.NITEMS, pl.pair, pl.NKC, pl.CPC};
   for (int i = 0; i < 32; ++i) out[i] = i < (int)(sizeof(v) / sizeof(v[0])) ? v[i] : 0;
   return I2CW_OK;
 }

@@ -17,13 +17,18 @@ constexpr int kMaxLanes = 128;  // UMMA M = 128 Winograd tiles per CTA (one TMEM
 // Everything the kernels need about one call; built by make_plan() in api.cu.
 struct Plan {
   int N, H, W, C, K, R, S;
+  int is_deconv;        // 1: deconvolution (U holds the rotated, channel-transposed filter)
+  int vol;              // 1: 3D convolution (x NDHWC, filter KTRSC): D, T, pad_d, OD, DB below
+  int D, T, pad_d, OD;  // input depth, filter depth taps, depth padding (kernel's view), output depth
+  int DB;               // 3D: depth blocks per image = ceil(OD / NI) (a tile block stacks NI output depths)
   int pad_h, pad_w;     // conv padding as seen by the kernel (deconv: R-1-pad, may be < 0)
   int P, Q;             // output height / width
   int m, alpha;         // F(m, S), alpha = m + S - 1
   int NT;               // output channels per CTA (UMMA N)
   int NB;               // ceil(K / NT)
-  int NCC;              // ceil(C / 8) channel chunks (8 fp32 = one tf32 UMMA K step)
-  int NKS;              // k-steps = NCC * R  (ks = cc * R + fh)
+  int NCC;              // chunks of the K loop: ceil(C / 8) channel chunks (8 fp32 = one tf32 UMMA K
+                        // step), times T depth taps in 3D (virtual chunk vc = cc * T + fd)
+  int NKS;              // k-steps = NCC * R  (ks = vc * R + fh)
   int T_r;              // Winograd tiles per output row = ceil(Q / m)
   int TS;               // tiles per row segment handled by one CTA
   int SEGS;             // segments per row = ceil(T_r / TS)
@@ -35,9 +40,11 @@ struct Plan {
   int PLANE;            // half an input stage (BOXB rounded up to 1024, halved)
   int tile_blocks;      // ceil(N / NI) * PB * SEGS
   int NFULL, NITEMS;    // work items: [0, NFULL) whole units; then 2 per tail unit (one per pass)
-  int GP, NPASS;        // points per pass (TMEM budget), passes = alpha / GP
-  int NUS;              // U pipeline stages (v1 kernel; v2 uses the template NS)
-  int OPITCH;           // (unused, kept for the debug plan layout)
+  int GP, NPASS;        // points per pass (TMEM budget), point groups = alpha / GP
+  int NKC, CPC;         // K-chunks (launches) of the K loop, channel chunks per K-chunk (bounded accumulation)
+  int CC0, CC1;         // this launch's channel chunks [CC0, CC1) (set per K-chunk launch)
+  int ACCUM;            // 1: every pass adds into y (a K-chunk after the first)
+  int NUS;              // U ring super-slots (KPS k-steps of GP points each)
   int OSB;              // bytes of one output staging buffer = NI*ROWS*TS*16*4 (TMA store box, 16 channels)
   int OSTRIDE;          // OSB rounded up to 1024 (swizzled TMA boxes need 1024-byte alignment)
   int NOB;              // output staging buffers per warpgroup (1..4)
@@ -55,7 +62,7 @@ struct Plan {
 // Points per TMEM pass: GP * NT = 256 accumulator columns (GP even, dividing alpha; the
 // other 256 columns hold the V slots).
 __host__ __device__ constexpr int gp_for(int alpha, int NT) {
-  return NT == 128 ? 2 : (NT == 64 ? 4 : (alpha % 8 == 0 ? 8 : 6));
+  return alpha <= 4 ? alpha : (NT == 128 ? 2 : (NT == 64 ? 4 : (alpha % 8 == 0 ? 8 : 6)));
 }
 // V slots (one k-step of GP points, hi + lo, each) next to the accumulators:
 // NS * GP * 16 <= 512 - GP * NT. NT = 128: 8 slots of 32 columns (two per warpgroup);
@@ -107,7 +114,7 @@ __host__ __device__ inline size_t u_offset_pair(int NT, int alpha, int nb, int N
 constexpr int kUTagBytes = 256;
 constexpr uint32_t kUMagic = 0x49324357u;  // "I2CW"
 struct UTag {
-  uint32_t magic, alpha, m, is_deconv, C, K, R, S, NT, NB, NCC, halves;
+  uint32_t magic, alpha, m, is_deconv, C, K, R, S, NT, NB, NCC, halves, T;  // T: depth taps (2D: 1)
 };
 
 #if defined(__CUDACC__)
@@ -209,6 +216,30 @@ __device__ __forceinline__ void tma_load_4d(void* smem_dst, const CUtensorMap* m
       : "memory");
 }
 // TMA: 4D tiled tensor store shared -> global (OOB elements of the box are not written)
+// 5D variants (3D convolution: C, W, H, D, N)
+__device__ __forceinline__ void tma_load_5d(void* smem_dst, const CUtensorMap* map, uint64_t* bar, int c0, int c1,
+                                            int c2, int c3, int c4) {
+  asm volatile(
+      "cp.async.bulk.tensor.5d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+      " [%0], [%1, {%2, %3, %4, %5, %6}], [%7];" ::"r"(smem_u32(smem_dst)),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "r"(c4), "r"(smem_u32(bar))
+      : "memory");
+}
+__device__ __forceinline__ void tma_store_5d(const CUtensorMap* map, const void* smem_src, int c0, int c1, int c2,
+                                             int c3, int c4) {
+  asm volatile("cp.async.bulk.tensor.5d.global.shared::cta.tile.bulk_group [%0, {%2, %3, %4, %5, %6}], [%1];" ::"l"(
+                   reinterpret_cast<uint64_t>(map)),
+               "r"(smem_u32(smem_src)), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "r"(c4)
+               : "memory");
+}
+__device__ __forceinline__ void tma_reduce_add_5d(const CUtensorMap* map, const void* smem_src, int c0, int c1,
+                                                  int c2, int c3, int c4) {
+  asm volatile(
+      "cp.reduce.async.bulk.tensor.5d.global.shared::cta.add.tile.bulk_group [%0, {%2, %3, %4, %5, %6}], [%1];" ::"l"(
+          reinterpret_cast<uint64_t>(map)),
+      "r"(smem_u32(smem_src)), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "r"(c4)
+      : "memory");
+}
 __device__ __forceinline__ void tma_store_4d(const CUtensorMap* map, const void* smem_src, int c0, int c1, int c2,
                                              int c3) {
   asm volatile("cp.async.bulk.tensor.4d.global.shared::cta.tile.bulk_group [%0, {%2, %3, %4, %5}], [%1];" ::"l"(

@@ -115,8 +115,12 @@ cudaError_t launch_filter_transform(const float* w, float* u, int C, int K, int 
 // dependent of the filter transform (it does not read U, so it may run concurrently with it),
 // lets the fused kernel launch at once, and waits for the filter transform's grid before it
 // exits, so the fused kernel's griddepcontrol.wait (on this grid) still covers U.
-__global__ void zero_tail_kernel(float* __restrict__ y, size_t count) {
+// wait_first: the previous kernel in the stream is not the library's own filter transform (the
+// pre-transformed path: whatever the caller ran last), so no store may happen before that grid
+// has completed -- the PDL rule that a dependent touches no memory before griddepcontrol.wait.
+__global__ void zero_tail_kernel(float* __restrict__ y, size_t count, int wait_first) {
   asm volatile("griddepcontrol.launch_dependents;");
+  if (wait_first) asm volatile("griddepcontrol.wait;" ::: "memory");
   const size_t tid = blockIdx.x * (size_t)blockDim.x + threadIdx.x, nth = (size_t)gridDim.x * blockDim.x;
   size_t head = 0;
   if ((reinterpret_cast<uintptr_t>(y) & 15) == 0) {
@@ -129,7 +133,7 @@ __global__ void zero_tail_kernel(float* __restrict__ y, size_t count) {
   asm volatile("griddepcontrol.wait;" ::: "memory");
 }
 
-cudaError_t launch_zero_tail(float* y, size_t count, cudaStream_t stream) {
+cudaError_t launch_zero_tail(float* y, size_t count, bool wait_first, cudaStream_t stream) {
   if (count == 0) return cudaSuccess;
   size_t want = (count / 4 + 255) / 256;
   const unsigned blocks = (unsigned)std::min<size_t>(std::max<size_t>(want, 1), 148 * 8);
@@ -142,7 +146,7 @@ cudaError_t launch_zero_tail(float* y, size_t count, cudaStream_t stream) {
   attr[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
-  cudaError_t e = cudaLaunchKernelEx(&cfg, zero_tail_kernel, y, count);
+  cudaError_t e = cudaLaunchKernelEx(&cfg, zero_tail_kernel, y, count, (int)wait_first);
   return e != cudaSuccess ? e : cudaGetLastError();
 }
 

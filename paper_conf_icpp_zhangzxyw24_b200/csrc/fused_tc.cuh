@@ -101,12 +101,33 @@ __device__ __forceinline__ float2 bt_dot2(const float2 (&d)[A][2], int p) {
     return acc;
   }
 }
-// 3xTF32 operand split of a channel pair: hi = v truncated to tf32 (exactly representable,
-// so the tensor core's own fp32->tf32 conversion mode does not matter), lo = v - hi (exact).
+// 3xTF32 operand split of a channel pair (reading R10): hi = v rounded to tf32 (11
+// significant bits, exactly representable, so the tensor core's own fp32->tf32 conversion does
+// not matter), lo = v - hi (exact in fp32; the tensor core drops lo's low bits, < 2^-22 |v|).
+// I2CW_SPLIT (build-time): 2 = Veltkamp splitting p = (2^13 + 1) v, hi = p - (p - v): round to
+// nearest (ties to even) in 3 packed FP ops, so lo takes either sign and its truncation by the
+// tensor core is unbiased (valid while |v| < FLT_MAX / 8193 ~ 4e34); 1 = the same rounding
+// (ties away) with integer ops, +5% kernel time (profiles/r02_ab_split.txt); 0 = truncation
+// (hi = v & ~0x1fff; lo one-signed: measured mean error on U[1,2] +60%).
+#ifndef I2CW_SPLIT
+#define I2CW_SPLIT 2
+#endif
+#ifndef I2CW_NO_TAGCHECK
+#define I2CW_NO_TAGCHECK 0      // experiment switch: 1 = no device-side U tag check
+#endif
 __device__ __forceinline__ void split_tf32x2(float2 v, float2& hi, float2& lo) {
+  const float2 neg1 = make_float2(-1.f, -1.f);
+#if I2CW_SPLIT == 2
+  const float2 p = __fmul2_rn(make_float2(8193.f, 8193.f), v);
+  hi = __ffma2_rn(neg1, __ffma2_rn(neg1, v, p), p);  // p - (p - v)
+#elif I2CW_SPLIT == 1
+  hi.x = __uint_as_float((__float_as_uint(v.x) + 0x1000u) & 0xFFFFE000u);
+  hi.y = __uint_as_float((__float_as_uint(v.y) + 0x1000u) & 0xFFFFE000u);
+#else
   hi.x = __uint_as_float(__float_as_uint(v.x) & 0xFFFFE000u);
   hi.y = __uint_as_float(__float_as_uint(v.y) & 0xFFFFE000u);
-  lo = __ffma2_rn(make_float2(-1.f, -1.f), hi, v);
+#endif
+  lo = __ffma2_rn(neg1, hi, v);
 }
 
 template <int M, int RW, int NT, bool PAIR>
@@ -141,7 +162,13 @@ struct TcCfg {
 // leader (rank 0) issues all MMAs; the peer's "relay" thread forwards "my V stage and U
 // half are in place" with one remote mbarrier arrive per k-step, and its epilogue's "D
 // read" with one per pass. Commits are multicast to the barriers of both CTAs.
-template <int M, int RW, int NT, bool PAIR>
+// VOL = true: 3D convolution ("expanding Stage1 Im2col to ND, while remaining
+// Stage2 unchanged"). x is [N][D][H][W][C], the filter [K][T][R][S][C] is used as the 2D filter
+// [K][T*R][S][C] (so U and the filter transform are the 2D ones with R' = T*R), and a "chunk" of
+// the K loop is a virtual chunk vc = cc * T + fd: channel chunk cc at depth tap fd, staged as one
+// input box at depth d0 - pad_d + fd. The NI slices a tile block stacks are consecutive OUTPUT
+// depths of one image (2D: consecutive images). Stage 2 (the 1D Winograd along W) is unchanged.
+template <int M, int RW, int NT, bool PAIR, bool VOL = false>
 __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
     fused_tc_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__ CUtensorMap ymap,
                     const __grid_constant__ Plan pl, const float* __restrict__ u) {
@@ -179,7 +206,7 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
   uint64_t* in_empty = in_full + NIS;   // [NIS]
   uint64_t* st_full = in_empty + NIS;   // [NSS]
   uint64_t* st_empty = st_full + NSS;   // [NSLOT]: one per V slot (its k-step's MMAs completed)
-  uint64_t* r_full = st_empty + NSLOT;  // [NSS]  (pair leader: the peer's super-stage relayed)
+  uint64_t* r_full = st_empty + NSLOT;  // [NSS]  (unused since the peer arrives directly; keeps the layout)
   uint64_t* d_full = r_full + NSS;      // [1]
   uint64_t* d_empty = d_full + 1;       // [1]
   uint64_t* u_full = d_empty + 1;       // [NUS]
@@ -205,7 +232,7 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
     else { const int h = it - pl.NFULL; I.ui = pl.NFULL + h / 2; I.pb = h % 2; I.pe = I.pb + 1; I.split = true; }
     return I;
   };
-  struct Unit { int nb, tb, seg, n, p0, crot; bool active; };
+  struct Unit { int nb, tb, seg, n, d0, p0, crot; bool active; };
   auto unit_at = [&](int ui) {
     Unit U;
     U.nb = ui % pl.NB;
@@ -214,15 +241,26 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
     U.seg = U.tb % pl.SEGS;
     const int tbr = U.tb / pl.SEGS;
     U.p0 = (tbr % pl.PB) * pl.ROWS;
-    U.n = (tbr / pl.PB) * pl.NI;
+    if constexpr (VOL) {  // image block = (image n, NI output depths from d0)
+      const int ib = tbr / pl.PB;
+      U.n = ib / pl.DB;
+      U.d0 = (ib - U.n * pl.DB) * pl.NI;
+    } else {
+      U.n = (tbr / pl.PB) * pl.NI;
+      U.d0 = 0;
+    }
     // Channel-chunk rotation: unit ui walks the chunks starting at crot, so SMs do not all
     // stream the same U image at the same time. Both CTAs of a pair rotate alike (their MMAs
     // consume the same k-step). The summation order is a function of the unit: results stay
     // run-to-run deterministic.
-    U.crot = (int)(((unsigned)ui * 5u) % (unsigned)pl.NCC);
+    U.crot = (int)(((unsigned)ui * 5u) % (unsigned)(pl.CC1 - pl.CC0));
     return U;
   };
-  const int NKS = pl.NKS;
+  // This launch's channel chunks [CC0, CC1) (the whole K loop, or one K-chunk of it: the host
+  // launches long K loops as several chunks, each accumulated from zero in TMEM and added into y
+  // by the TMA reduce-add). NKS = this launch's k-steps.
+  const int CC0 = pl.CC0, NCCL = pl.CC1 - pl.CC0;
+  const int NKS = NCCL * pl.R;
   const int NKSP = (NKS + KPS - 1) / KPS * KPS;   // k-steps per pass padded to whole super-stages
   constexpr int PROD_WARP = NWG * 4, UPROD_WARP = NWG * 4 + 1, ISS_WARP0 = NWG * 4 + 2;
 
@@ -231,13 +269,15 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
     // per-thread arrivals on one barrier word serialise in the shared-memory atomic unit
     for (int i = 0; i < NIS; ++i) { mbar_init(&in_full[i], 1); mbar_init(&in_empty[i], NWG * 4); }
     for (int i = 0; i < NSS; ++i) {
-      mbar_init(&st_full[i], KPS * 4);  // the 4 warps of each of the KPS warpgroups of this super-stage
-      mbar_init(&r_full[i], 1);
+      // the 4 warps of each of the KPS warpgroups of this super-stage; a pair leader also counts
+      // the peer's 4 x KPS warps, which arrive remotely (no relay thread on the V path)
+      mbar_init(&st_full[i], KPS * 4 * (PAIR && rank == 0 ? 2 : 1));
     }
     for (int i = 0; i < NSLOT; ++i) mbar_init(&st_empty[i], NISS);
-    for (int i = 0; i < NUS; ++i) { mbar_init(&u_full[i], 1); mbar_init(&u_empty[i], NISS); }
+    // pair leader's U slot: its own expect_tx arrive + the peer's "my half landed" arrive
+    for (int i = 0; i < NUS; ++i) { mbar_init(&u_full[i], PAIR && rank == 0 ? 2 : 1); mbar_init(&u_empty[i], NISS); }
     mbar_init(d_full, NISS);
-    mbar_init(d_empty, NWG * 4 + (PAIR && rank == 0 ? 1 : 0));
+    mbar_init(d_empty, NWG * 4 * (PAIR && rank == 0 ? 2 : 1));  // pair: the peer's warps arrive remotely
     fence_mbar_init();
   }
   if (warp == ISS_WARP0) {  // the first issuer warp owns the TMEM allocation
@@ -275,6 +315,18 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
     // (kg = PASS * NKSP + cc * R + fh): the four warpgroups' transforms interleave on the
     // SMSPs, each k-step's full V (GP points x 8 channels, hi + lo) written by one warpgroup.
     const uint32_t vbase0 = lane_addr + VCOL;
+    // "V of this k-step stored" / "accumulators read": local arrive, or for the pair peer a remote
+    // arrive on the leader's barrier (the leader's MMAs read this CTA's TMEM; tcgen05.wait::st has
+    // completed the stores before the arrive)
+    const uint32_t st_full_lead = PAIR ? mapa_shared(st_full, 0) : 0u, d_empty_lead = PAIR ? mapa_shared(d_empty, 0) : 0u;
+    auto arrive_st_full = [&](int idx) {
+      if (PAIR && rank == 1) mbar_arrive_remote(st_full_lead + 8u * (uint32_t)idx);
+      else mbar_arrive(&st_full[idx]);
+    };
+    auto arrive_d_empty = [&]() {
+      if (PAIR && rank == 1) mbar_arrive_remote(d_empty_lead);
+      else mbar_arrive(d_empty);
+    };
     auto wait_slot = [&](int kg) {  // this slot's previous k-step consumed (tcgen05.commit per k-step)
       const int use = kg / NSLOT;
       if (use > 0) mbar_wait_tc<PAIR>(&st_empty[kg & (NSLOT - 1)], (use - 1) & 1);
@@ -289,7 +341,7 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
       if (PASS < I.pb || PASS >= I.pe) return;
       const int gpass = pc++;
       const int kgp = gpass * NKSP;  // global index of this pass's first k-step
-      for (int cc = 0; cc < pl.NCC; ++cc) {
+      for (int cc = 0; cc < NCCL; ++cc) {
         const int kb = kgp + cc * pl.R;  // global index of the chunk's first k-step
         trace_rec(pl.trace, 19 + g, PASS * pl.NCC + cc, l == 0);
         // every warpgroup waits for every chunk (also one it has no k-step in, R < NWG) so
@@ -369,7 +421,7 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
           tmem_wait_st();
           tc_fence_before();
           __syncwarp();
-          if (lane32 == 0) mbar_arrive(&st_full[(kg / KPS) % NSS]);
+          if (lane32 == 0) arrive_st_full((kg / KPS) % NSS);
           trace_rec(pl.trace, 8 + g, kg / NWG, l == 0);
         }
         __syncwarp();
@@ -384,7 +436,7 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
         wait_slot(kg);
         tc_fence_before();
         __syncwarp();
-        if (lane32 == 0) mbar_arrive(&st_full[(kg / KPS) % NSS]);
+        if (lane32 == 0) arrive_st_full((kg / KPS) % NSS);
       }
       // ---------- epilogue of this pass: y (+)= A^T M via shared memory + TMA ----------
       trace_rec(pl.trace, 27, 2 * gpass, l == 0 && g == 0);
@@ -403,7 +455,7 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
       if (ABL(4)) {  // DEBUG timing ablation: release the accumulators, no y
         tc_fence_before();
         __syncwarp();
-        if (lane32 == 0) mbar_arrive(d_empty);
+        if (lane32 == 0) arrive_d_empty();
       } else {
         float mv[GP][CPW];
 #pragma unroll
@@ -413,7 +465,8 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
         tmem_wait_ld();
         tc_fence_before();
         __syncwarp();
-        if (lane32 == 0) mbar_arrive(d_empty);  // accumulators read: the next pass may overwrite them
+        if (lane32 == 0) arrive_d_empty();  // accumulators read: the next pass may overwrite them
+        trace_rec(pl.trace, 28, 128 + 2 * gpass, l == 0 && g == 0);
         static_for<GP / 2>([&](auto Q_) {  // pair (a, a+1): AT[i][a+1] = (-1)^i AT[i][a]
           constexpr int idx0 = PASS * GP + 2 * (int)Q_;
           constexpr int tl0 = 2 * (int)Q_;
@@ -429,6 +482,7 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
         });
         if (l == 0) bulk_wait_group_read_dyn(pl.NOB - 1);  // buffer 0: previous pass's stores
         named_bar_sync(1 + g, 128);
+        trace_rec(pl.trace, 28, 129 + 2 * gpass, l == 0 && g == 0);
         static_for<M>([&](auto I_) {
           constexpr int i = I_;
           const int ob = i % pl.NOB;
@@ -463,16 +517,26 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
             });
             if (has_slot && !(ABL(64))) stg[j ^ oswz] = make_float4(o[0].x, o[0].y, o[1].x, o[1].y);
           }
+          trace_rec(pl.trace, 27, 66 + 4 * (gpass * M + i), l == 0 && g == 0);
           fence_proxy_async_smem();
           // the store that last read the next column's buffer (column i + 1 - NOB) must be done
           if (l == 0) bulk_wait_group_read_dyn(pl.NOB - 2);
+          trace_rec(pl.trace, 27, 67 + 4 * (gpass * M + i), l == 0 && g == 0);
           named_bar_sync(1 + g, 128);
           trace_rec(pl.trace, 27, 65 + 4 * (gpass * M + i), l == 0 && g == 0);
           if (l == 0) {
             const float* box = ostage + (size_t)ob * (pl.OSTRIDE / 4);
             if (U.active && !(ABL(32))) {  // DEBUG ablation 32: no y stores
-              if (PASS == 0 && !I.split) tma_store_4d(&ymap, box, U.nb * NT + cbase, qbase + i, U.p0, U.n);
-              else tma_reduce_add_4d(&ymap, box, U.nb * NT + cbase, qbase + i, U.p0, U.n);
+              // first pass of the first K-chunk stores; others add (DEBUG ablation 512: stores only)
+              if constexpr (VOL) {
+                if (PASS == 0 && !I.split && !pl.ACCUM)
+                  tma_store_5d(&ymap, box, U.nb * NT + cbase, qbase + i, U.p0, U.d0, U.n);
+                else tma_reduce_add_5d(&ymap, box, U.nb * NT + cbase, qbase + i, U.p0, U.d0, U.n);
+              } else {
+                if ((PASS == 0 && !I.split && !pl.ACCUM) || ABL(512))
+                  tma_store_4d(&ymap, box, U.nb * NT + cbase, qbase + i, U.p0, U.n);
+                else tma_reduce_add_4d(&ymap, box, U.nb * NT + cbase, qbase + i, U.p0, U.n);
+              }
             }
             bulk_commit_group();
           }
@@ -500,15 +564,20 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
       const int wstart = U.seg * pl.TS * M - pl.pad_w;
       const int hstart = U.p0 - pl.pad_h;
       for (int pass = I.pb; pass < I.pe; ++pass) {
-        for (int cc = 0; cc < pl.NCC; ++cc) {
+        for (int cc = 0; cc < NCCL; ++cc) {
           if (!first) mbar_wait(&in_empty[ist], iph ^ 1);
           uint8_t* dst = in_smem + (size_t)ist * 2 * inplane;
-          const int ca = cc + U.crot < pl.NCC ? cc + U.crot : cc + U.crot - pl.NCC;  // actual chunk
+          const int ca = CC0 + (cc + U.crot < NCCL ? cc + U.crot : cc + U.crot - NCCL);  // actual chunk
           if (ABL(16)) {  // DEBUG timing ablation: no input rows (stage reused as is)
             mbar_arrive(&in_full[ist]);
           } else {
             mbar_expect_tx(&in_full[ist], (uint32_t)pl.BOXB);
-            tma_load_4d(dst, &xmap, &in_full[ist], ca * 8, wstart, hstart, U.n);
+            if constexpr (VOL) {  // virtual chunk ca = channel chunk * T + depth tap
+              const int cch = ca / pl.T, fd = ca - cch * pl.T;
+              tma_load_5d(dst, &xmap, &in_full[ist], cch * 8, wstart, hstart, U.d0 - pl.pad_d + fd, U.n);
+            } else {
+              tma_load_4d(dst, &xmap, &in_full[ist], ca * 8, wstart, hstart, U.n);
+            }
           }
           if (++ist == NIS) { ist = 0; iph ^= 1; first = 0; }
         }
@@ -520,6 +589,15 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
     // ================= U (transformed filter) super-slot ring =================
     if (lane32 == 0) {
       asm volatile("griddepcontrol.wait;" ::: "memory");  // U written by the previous kernel
+      // the device tag in front of U must describe this call (the host validated a copy of it;
+      // a stale host copy for a reused address must not run a mismatched filter silently)
+      if (!I2CW_NO_TAGCHECK && blockIdx.x == 0) {
+        const UTag* tg = reinterpret_cast<const UTag*>(reinterpret_cast<const uint8_t*>(u) - kUTagBytes);
+        if (tg->magic != kUMagic || (int)tg->alpha != A || (int)tg->m != M || (int)tg->is_deconv != pl.is_deconv ||
+            (int)tg->C != pl.C || (int)tg->K != pl.K || (int)tg->R != pl.R || (int)tg->S != RW ||
+            (int)tg->NT != NT || (int)tg->halves != (PAIR ? 2 : 1) || (int)tg->T != pl.T)
+          __trap();
+      }
       const size_t kstride = (size_t)A * 2 * NT * 8;  // floats per k-step (both layouts)
       int us = 0, uph = 0, first = 1;
       for (int it = unit0; it < NITEMS; it += ustride) {
@@ -527,8 +605,8 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
       const Unit U = unit_at(I.ui);
       for (int pass = I.pb; pass < I.pe; ++pass) {
         // this CTA's B rows of the pass's GP points, hi+lo, contiguous (pair: its N half)
-        const float* src0 = u + (PAIR ? u_offset_pair(NT, A, U.nb, NKS, 0, (int)rank, pass * GP)
-                                      : u_offset(NT, A, U.nb, NKS, 0, pass * GP, 0));
+        const float* src0 = u + (PAIR ? u_offset_pair(NT, A, U.nb, pl.NKS, 0, (int)rank, pass * GP)
+                                      : u_offset(NT, A, U.nb, pl.NKS, 0, pass * GP, 0));
         for (int kl0 = 0; kl0 < NKSP; kl0 += KPS) {
           trace_rec(pl.trace, 30, pass * NKSP + kl0);
           if (!first) mbar_wait_tc<PAIR>(&u_empty[us], uph ^ 1);  // completed by tcgen05.commit
@@ -538,7 +616,7 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
           mbar_expect_tx(&u_full[us], (uint32_t)nreal * ub);
           for (int pos = 0; pos < nreal; ++pos) {
             const int kl = kl0 + pos, cc = kl / pl.R, fh = kl - cc * pl.R;
-            const int ca = cc + U.crot < pl.NCC ? cc + U.crot : cc + U.crot - pl.NCC;
+            const int ca = CC0 + (cc + U.crot < NCCL ? cc + U.crot : cc + U.crot - NCCL);
             bulk_load(u_smem + (size_t)us * USBYTES + (size_t)pos * UBYTES, src0 + (size_t)(ca * pl.R + fh) * kstride,
                       ub, &u_full[us]);
           }
@@ -566,9 +644,13 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
         }
         for (int kl0 = 0; kl0 < NKSP; kl0 += KPS, ++sgi) {
           trace_rec(pl.trace, 29, sgi, iss == 0 && lane32 == 0);
-          mbar_wait(&st_full[ss], sph);
-          mbar_wait(&u_full[us], uph);
-          if constexpr (PAIR) mbar_wait_cluster(&r_full[ss], sph);  // the peer's V + U half
+          if constexpr (PAIR) {  // both CTAs' V (peer arrivals are remote) and both U halves
+            mbar_wait_cluster(&st_full[ss], sph);
+            mbar_wait_cluster(&u_full[us], uph);
+          } else {
+            mbar_wait(&st_full[ss], sph);
+            mbar_wait(&u_full[us], uph);
+          }
           tc_fence_after();
           trace_rec(pl.trace, 16, sgi, iss == 0 && lane32 == 0);
           if (!(ABL(2))) {  // DEBUG timing ablation: skip the MMAs (commits still signal)
@@ -621,25 +703,19 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
       }
       }  // units
     } else if (PAIR && lane32 == 0 && rank == 1 && iss == 0) {
-      // ===== pair peer relay: forward this CTA's super-stage readiness / D drain =====
-      const uint32_t lead_rfull = mapa_shared(r_full, 0), lead_dempty = mapa_shared(d_empty, 0);
-      int ss = 0, sph = 0, us = 0, uph = 0, sgi = 0, gpass = 0;
+      // ===== pair peer: forward "my U half landed" to the leader's U slot =====
+      // (off the critical path: the U ring runs several super-stages ahead; V readiness and the D
+      // drain are signalled by the peer's transform warps themselves, remotely)
+      const uint32_t lead_ufull = mapa_shared(u_full, 0);
+      int us = 0, uph = 0;
       for (int it = unit0; it < NITEMS; it += ustride) {
       const Item I = item_at(it);
-      for (int pass = I.pb; pass < I.pe; ++pass, ++gpass) {
-        for (int kl0 = 0; kl0 < NKSP; kl0 += KPS, ++sgi) {
-          mbar_wait(&st_full[ss], sph);
+      for (int pass = I.pb; pass < I.pe; ++pass) {
+        for (int kl0 = 0; kl0 < NKSP; kl0 += KPS) {
           mbar_wait(&u_full[us], uph);
-          tc_fence_after();
-          mbar_arrive_remote(lead_rfull + 8u * ss);
-          trace_rec(pl.trace, 17, sgi);
-          if (++ss == NSS) { ss = 0; sph ^= 1; }
+          mbar_arrive_remote(lead_ufull + 8u * (uint32_t)us);
           if (++us == NUS) { us = 0; uph ^= 1; }
         }
-        // this CTA's epilogue has read its D: the leader may overwrite it
-        mbar_wait(d_empty, gpass & 1);
-        tc_fence_after();
-        mbar_arrive_remote(lead_dempty);
       }
       }  // units
     }
@@ -672,11 +748,11 @@ inline int persistent_ctas(int units, int per) {
   return (units < slots ? units : slots) * per;
 }
 
-template <int M, int RW, int NT, bool PAIR>
+template <int M, int RW, int NT, bool PAIR, bool VOL = false>
 static cudaError_t launch_tc_t(const CUtensorMap& xmap, const CUtensorMap& ymap, const Plan& pl, const float* u,
                                cudaStream_t stream) {
   using Cfg = TcCfg<M, RW, NT, PAIR>;
-  auto kern = fused_tc_kernel<M, RW, NT, PAIR>;
+  auto kern = fused_tc_kernel<M, RW, NT, PAIR, VOL>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, pl.smem_bytes);
   if (e != cudaSuccess) return e;
   if constexpr (PAIR) {

@@ -102,3 +102,36 @@ def test_invalid_arguments_rejected_before_cuda():
     assert L.i2cw_deconv2d_nhwc(*args(S=12), fake, fake, fake, None) == i2cw.I2CW_EUNSUPPORTED
     assert L.i2cw_filter_bytes(8, 8, 3, 11) == 0
     assert L.i2cw_filter_bytes(64, 64, 3, 3) == 256 + 2 * 8 * 64 * 3 * 64 * 4
+    # argument order (K, C, R, S) as SURVEY.md §8(b): K = 40 -> NT = 64 (one block), C = 16 -> 2 chunks
+    assert L.i2cw_filter_bytes(40, 16, 3, 3) == 256 + 2 * 8 * 64 * 3 * 16 * 4
+    # K = 16 -> NT = 32, C = 40 -> 5 chunks
+    assert L.i2cw_filter_bytes(16, 40, 3, 3) == 256 + 2 * 8 * 32 * 3 * 40 * 4
+    assert i2cw.filter_bytes(16, 40, 3, 3) == L.i2cw_filter_bytes(16, 40, 3, 3)
+
+
+def test_planner_concurrent_shapes():
+    """Two host threads planning different shapes at the same time see the same plans as a
+    single thread (the plan memo and the transform-table memo are shared, mutex-guarded)."""
+    import threading
+    shapes = [("conv", 2, 13, 37, 16, 40, r, r, r // 2, r // 2) for r in range(2, 10)] + \
+             [("deconv", 3, 11, 23, 12, 12, r, r, r - 1, 0) for r in range(2, 10)]
+    ref = [i2cw.debug_plan(*s) for s in shapes]
+    errs = []
+
+    def work(order):
+        try:
+            for _ in range(20):
+                for i in order:
+                    assert i2cw.debug_plan(*shapes[i]) == ref[i]
+                    at, g, bt = i2cw.transform_matrices(*i2cw.plan(shapes[i][7])[:1], shapes[i][7])
+                    assert len(g) == i2cw.plan(shapes[i][7])[1]
+        except Exception as e:  # pragma: no cover - reported below
+            errs.append(e)
+
+    ts = [threading.Thread(target=work, args=(list(range(len(shapes))),)),
+          threading.Thread(target=work, args=(list(reversed(range(len(shapes)))),))]
+    for t in ts:
+        t.start()
+    for t in ts:
+        t.join()
+    assert not errs, errs

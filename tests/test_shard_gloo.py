@@ -53,6 +53,32 @@ def _worker(rank, world, port):
         dist.destroy_process_group()
 
 
+def _bench_worker(rank, world, port):
+    """bench.py's strong-scaling split: each rank draws ITS images with bench.make_x_device
+    (per-image seeds), the shards gathered over the process group equal the unsharded batch,
+    and the MAX-over-ranks time reduction is what the whole-job value divides by."""
+    import bench
+    dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank, world_size=world)
+    try:
+        n0, n1 = shard_range(N_GLOBAL, world, rank)
+        xs = bench.make_x_device(n0, n1, H, W, C, torch.device("cpu"))
+        x_all = gather_rows(xs)
+        if rank == 0:
+            assert torch.equal(x_all, bench.make_x_device(0, N_GLOBAL, H, W, C, torch.device("cpu")))
+        t = max_over_ranks([0.5 + rank])
+        assert t == [0.5 + world - 1]
+        cfg = ("conv", N_GLOBAL, H, W, C, K, 3, 3, 1, 1, "")
+        # whole-job throughput: all N_GLOBAL images over the slowest rank's time
+        assert bench.direct_flops(cfg) == 2.0 * N_GLOBAL * H * W * C * K * 9
+    finally:
+        dist.destroy_process_group()
+
+
+def test_bench_strong_scaling_split_gloo_world2():
+    os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+    mp.spawn(_bench_worker, args=(2, _free_port()), nprocs=2, join=True)
+
+
 def test_shard_range_balanced_cover():
     for n in (0, 1, 5, 8, 13, 256):
         for world in (1, 2, 3, 4, 8):

@@ -90,11 +90,16 @@ for name in sys.argv[1:] or ["cfg2"]:
             if lo_ <= tt < lo_ + 12000:
                 print(f"   {tt:8d} (+{tt - prev if prev is not None else 0:5d}) {s}"); prev = tt
     e27 = T2[0][27]
+    e28 = T2[0][28]
     if (e27[64:] >= 0).any():
-        print("epilogue columns (WG0 thread 0): col: bulk-wait, bar1, compute+STS+bar2, to next")
-        prev = None
+        print("epilogue per pass (WG0 thread 0): d_full wait, TMEM ld -> d_empty, pair sums + pre-bar")
+        for gp in range(0, 24):
+            if e27[2 * gp] < 0 or e28[128 + 2 * gp] < 0: continue
+            print(f"   pass {gp}: d_full wait {e27[2*gp+1]-e27[2*gp]}  tmem ld {e28[128+2*gp]-e27[2*gp+1]}  pre {e28[129+2*gp]-e28[128+2*gp]}")
+        print("epilogue columns (WG0 thread 0): col: compute+STS, fence+bulk-wait, bar, store issue -> next col")
         for c in range(0, 60):
             b = 64 + 4 * c
-            if e27[b] < 0: continue
-            nxt = e27[b + 4] if e27[b + 4] >= 0 else -1
-            print(f"   {c:3d} t={e27[b]} wait {e27[b+1]-e27[b]} bar1 {e27[b+2]-e27[b+1]} body {e27[b+3]-e27[b+2]} next {nxt-e27[b+3] if nxt>=0 else None}")
+            if b + 3 >= 512 or e27[b] < 0: continue
+            nxt = e27[b + 4] if b + 4 < 512 and e27[b + 4] >= 0 else -1
+            print(f"   {c:3d} t={e27[b]} compute+sts {e27[b+2]-e27[b]} fence+wait {e27[b+3]-e27[b+2]} bar {e27[b+1]-e27[b+3]} "
+                  f"-> next {nxt-e27[b+1] if nxt>=0 else None}")
