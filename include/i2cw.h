@@ -103,6 +103,24 @@ I2CW_API int i2cw_deconv2d_nhwc(int N, int H, int W, int C, int K, int R, int S,
                        const float* x, const float* w, float* y, i2cw_stream_t stream);
 
 /*
+ * Precision modes ("1xTF32 with looser tolerance").
+ *   I2CW_PREC_3XTF32 (default of every other call): hi*hi + hi*lo + lo*hi tf32 products,
+ *     |y - y_exact| <= 1e-4 * sum|x||w| per element.
+ *   I2CW_PREC_1XTF32: one tf32 product per Winograd point (V and U rounded to nearest tf32,
+ *     a third of the tensor work); tolerance |y - y_exact| <= 1e-2 * sum|x||w| (each product's
+ *     relative error <= 2^-10, amplified <= ~10x by the alpha <= 12 transforms; measured max
+ *     3.1e-3, profiles/r02_precision.txt; reading R17).
+ * i2cw_conv2d_nhwc_prec: the 2D conv (is_deconv = 0, w KRSC) or deconv (is_deconv = 1, w CRSK)
+ * with the given precision; otherwise as i2cw_conv2d_nhwc / i2cw_deconv2d_nhwc.
+ * EINVAL for an unknown precision.
+ */
+#define I2CW_PREC_3XTF32 0
+#define I2CW_PREC_1XTF32 1
+I2CW_API int i2cw_conv2d_nhwc_prec(int precision, int is_deconv, int N, int H, int W, int C, int K, int R, int S,
+                                   int pad_h, int pad_w, const float* x, const float* w, float* y,
+                                   i2cw_stream_t stream);
+
+/*
  * 3D convolution (Im2col-Winograd "can be applied to ND convolution, by
  * expanding Stage1 Im2col to ND, while remaining Stage2 unchanged"): the 1D F(m, S) Winograd
  * runs along W exactly as in 2D; the K loop of the channel contraction runs over (c, depth tap
@@ -182,9 +200,11 @@ I2CW_API int i2cw_set_device(int device);
 
 /*
  * Host-side introspection (no GPU needed).
- * i2cw_plan: the Winograd choice for filter width S: m outputs, alpha = m+S-1
- *   states, and the alpha = 16 point set (0 paper, 1 alt; reading R7).
- *   Returns I2CW_EUNSUPPORTED for S outside [2, 9].
+ * i2cw_plan: the Winograd choice for filter width S and C input channels: m outputs,
+ *   alpha = m+S-1 states, and the alpha = 16 point set (0 paper, 1 alt; reading R7).
+ *   S = 2: Gamma4(3,2); S = 3: Gamma4(2,3) when C >= 256, else Gamma8(6,3); S = 4..7: Gamma8;
+ *   S = 8, 9: alpha = 12 (measured selection, reading R8). The 3D and 1xTF32 calls use
+ *   alpha = 8 for S = 2, 3. Returns I2CW_EUNSUPPORTED for S outside [2, 9], EINVAL for C <= 0.
  * i2cw_transform_matrices_rational: the exact Cook-Toom matrices of F(m, r)
  *   (§5.3, Figure 5) as int64 numerator/denominator
  *   pairs, row-major: AT (m x alpha), G (alpha x r), BT (alpha x alpha), with
@@ -192,7 +212,7 @@ I2CW_API int i2cw_set_device(int device);
  *   Each output array must hold the matrix's element count; returns I2CW_EINVAL
  *   on bad arguments and I2CW_EUNSUPPORTED if an entry does not fit in int64.
  */
-I2CW_API int i2cw_plan(int S, int* m, int* alpha, int* point_set);
+I2CW_API int i2cw_plan(int S, int C, int* m, int* alpha, int* point_set);
 I2CW_API int i2cw_transform_matrices_rational(int m, int r, int point_set, int64_t* at_num, int64_t* at_den,
                                      int64_t* g_num, int64_t* g_den, int64_t* bt_num, int64_t* bt_den);
 

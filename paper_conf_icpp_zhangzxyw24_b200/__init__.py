@@ -26,7 +26,13 @@ PUBLIC_SYMBOLS = (
     "i2cw_filter_transform", "i2cw_conv2d_nhwc_pretransformed", "i2cw_deconv2d_nhwc_pretransformed",
     "i2cw_conv2d_nhwc_host", "i2cw_set_device", "i2cw_plan", "i2cw_transform_matrices_rational",
     "i2cw_conv3d_ndhwc", "i2cw_deconv3d_ndhwc", "i2cw_conv2d_nchw", "i2cw_deconv2d_nchw",
+    "i2cw_conv2d_nhwc_prec",
 )
+
+#: precision modes of i2cw_conv2d_nhwc_prec (include/i2cw.h)
+PRECISIONS = {"3xtf32": 0, "1xtf32": 1}
+#: per-element tolerance (x sum|x||w|) each precision mode guarantees
+TOLERANCE = {"3xtf32": 1e-4, "1xtf32": 1e-2}
 
 
 class I2CWError(RuntimeError):
@@ -51,6 +57,8 @@ def lib():
             f = getattr(L, name)
             f.argtypes = [I] * 9 + [P, P, P, P]
             f.restype = I
+        L.i2cw_conv2d_nhwc_prec.argtypes = [I] * 11 + [P, P, P, P]
+        L.i2cw_conv2d_nhwc_prec.restype = I
         for name in ("i2cw_conv2d_nchw", "i2cw_deconv2d_nchw"):
             f = getattr(L, name)
             f.argtypes = [I] * 9 + [P, P, P, P]
@@ -67,7 +75,7 @@ def lib():
         L.i2cw_conv2d_nhwc_host.restype = I
         L.i2cw_set_device.argtypes = [I]
         L.i2cw_set_device.restype = I
-        L.i2cw_plan.argtypes = [I, P, P, P]
+        L.i2cw_plan.argtypes = [I, I, P, P, P]
         L.i2cw_plan.restype = I
         L.i2cw_transform_matrices_rational.argtypes = [I, I, I] + [P] * 6
         L.i2cw_transform_matrices_rational.restype = I
@@ -121,9 +129,9 @@ def out_shape(kind, N, H, W, K, R, S, pad_h, pad_w):
     return (N, H + R - 1 - 2 * pad_h, W + S - 1 - 2 * pad_w, K)
 
 
-def conv2d_nhwc(x, w, pad_h, pad_w, out=None, stream=None):
-    """y = conv(x, w) (cross-correlation, zero padding); x [N,H,W,C], w [K,R,S,C] -> y [N,P,Q,K]."""
-    import torch
+def conv2d_nhwc(x, w, pad_h, pad_w, out=None, stream=None, precision="3xtf32"):
+    """y = conv(x, w) (cross-correlation, zero padding); x [N,H,W,C], w [K,R,S,C] -> y [N,P,Q,K].
+    precision: "3xtf32" (fp32 accuracy, default) or "1xtf32" (one tf32 product, TOLERANCE)."""
     _check_tensor(x, "x"); _check_tensor(w, "w")
     N, H, W, C = x.shape
     K, R, S, C2 = w.shape
@@ -132,14 +140,18 @@ def conv2d_nhwc(x, w, pad_h, pad_w, out=None, stream=None):
     if w.device != x.device:
         raise ValueError("x and w must be on the same device")
     y = _out(out, out_shape("conv", N, H, W, K, R, S, pad_h, pad_w), x)
+    if precision != "3xtf32":
+        _check("i2cw_conv2d_nhwc_prec", lib().i2cw_conv2d_nhwc_prec(
+            PRECISIONS[precision], 0, N, H, W, C, K, R, S, pad_h, pad_w, x.data_ptr(), w.data_ptr(), y.data_ptr(),
+            _stream_ptr(stream)))
+        return y
     _check("i2cw_conv2d_nhwc", lib().i2cw_conv2d_nhwc(N, H, W, C, K, R, S, pad_h, pad_w, x.data_ptr(), w.data_ptr(),
                                                       y.data_ptr(), _stream_ptr(stream)))
     return y
 
 
-def deconv2d_nhwc(x, w, pad_h, pad_w, out=None, stream=None):
+def deconv2d_nhwc(x, w, pad_h, pad_w, out=None, stream=None, precision="3xtf32"):
     """Transposed conv; x [N,H,W,C], w [C,R,S,K] -> y [N,P,Q,K], P = H+R-1-2 pad_h."""
-    import torch
     _check_tensor(x, "x"); _check_tensor(w, "w")
     N, H, W, C = x.shape
     C2, R, S, K = w.shape
@@ -148,6 +160,11 @@ def deconv2d_nhwc(x, w, pad_h, pad_w, out=None, stream=None):
     if w.device != x.device:
         raise ValueError("x and w must be on the same device")
     y = _out(out, out_shape("deconv", N, H, W, K, R, S, pad_h, pad_w), x)
+    if precision != "3xtf32":
+        _check("i2cw_conv2d_nhwc_prec", lib().i2cw_conv2d_nhwc_prec(
+            PRECISIONS[precision], 1, N, H, W, C, K, R, S, pad_h, pad_w, x.data_ptr(), w.data_ptr(), y.data_ptr(),
+            _stream_ptr(stream)))
+        return y
     _check("i2cw_deconv2d_nhwc", lib().i2cw_deconv2d_nhwc(N, H, W, C, K, R, S, pad_h, pad_w, x.data_ptr(),
                                                           w.data_ptr(), y.data_ptr(), _stream_ptr(stream)))
     return y
@@ -283,9 +300,10 @@ def conv2d_nhwc_host(x, w, pad_h, pad_w, is_deconv=False, out=None, stream=None)
     return y
 
 
-def plan(S):
+def plan(S, C=64):
+    """(m, alpha, point_set) the library uses for filter width S with C input channels."""
     m, a, ps = ctypes.c_int(), ctypes.c_int(), ctypes.c_int()
-    _check("i2cw_plan", lib().i2cw_plan(S, ctypes.byref(m), ctypes.byref(a), ctypes.byref(ps)))
+    _check("i2cw_plan", lib().i2cw_plan(S, C, ctypes.byref(m), ctypes.byref(a), ctypes.byref(ps)))
     return m.value, a.value, ps.value
 
 

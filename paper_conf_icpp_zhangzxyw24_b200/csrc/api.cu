@@ -55,17 +55,26 @@ bool alpha16_override() {
   static const bool on = [] { const char* e = getenv("I2CW_ALPHA16"); return e && e[0] == '1'; }();
   return on;
 }
-// I2CW_ALPHA=4 (experiments): Gamma4(3,2) / Gamma4(2,3) for S = 2, 3
-bool alpha4_override() {
-  static const bool on = [] { const char* e = getenv("I2CW_ALPHA"); return e && atoi(e) == 4; }();
-  return on;
+// Per (S, C) choice of F(m, S) -- a function of the filter only, so a pre-transformed U fits
+// every call with that filter. r = 4..7 follow the paper's Gamma_8 choices (Table 2,
+// PAPER.md:3968-3984); r = 8, 9 use alpha = 12 (reading R7). For S = 2 and S = 3 the
+// paper's Gamma_4 variants were measured against Gamma_8 on B200
+// (profiles/r02_variant_sweep.txt): F(3,2) alpha = 4 beats F(7,2) alpha = 8 by 31% (cfg3-r2), and
+// F(2,3) alpha = 4 beats F(6,3) alpha = 8 by ~6% at C >= 256 (cfg5b c256/c512, with CTA pairs)
+// but loses 15% on cfg2 and 2.5% at C = 128: one pass (no reduce-add of a second point group)
+// against 1.5x the tensor work. I2CW_ALPHA=4 / 8 forces the alpha = 4 / 8 variant for S = 2, 3.
+int alpha_env() {
+  static const int v = [] { const char* e = getenv("I2CW_ALPHA"); return e ? atoi(e) : 0; }();
+  return v;
 }
-bool choose(int S, Choice* c) {
+bool choose(int S, int C, Choice* c) {
   if (alpha16_override() && S >= 7 && S <= 9) { *c = {17 - S, 16, 1}; return true; }
-  if (alpha4_override() && (S == 2 || S == 3)) { *c = {5 - S, 4, 0}; return true; }
+  if (S == 2 || S == 3) {
+    const bool a4 = alpha_env() == 4 || (alpha_env() != 8 && (S == 2 || C >= 256));
+    *c = a4 ? Choice{5 - S, 4, 0} : Choice{9 - S, 8, 0};
+    return true;
+  }
   switch (S) {
-    case 2: *c = {7, 8, 0}; return true;
-    case 3: *c = {6, 8, 0}; return true;
     case 4: *c = {5, 8, 0}; return true;
     case 5: *c = {4, 8, 0}; return true;
     case 6: *c = {3, 8, 0}; return true;
@@ -140,20 +149,22 @@ int num_sms() {
 // Build the launch plan. Returns I2CW_OK or an error code.
 // vol = 1: 3D convolution (D, T, pad_d); 2D calls pass D = T = 1, pad_d = 0, vol = 0.
 int make_plan_uncached(int N, int D, int H, int W, int C, int K, int T, int R, int S, int pad_d, int pad_h, int pad_w,
-                       int is_deconv, int vol, Plan* out) {
+                       int is_deconv, int vol, int prec, Plan* out) {
   Plan pl;
   std::memset(&pl, 0, sizeof(pl));
   if (N <= 0 || D <= 0 || H <= 0 || W <= 0 || C <= 0 || K <= 0 || T <= 0 || R <= 0 || S <= 0 || pad_d < 0 ||
       pad_h < 0 || pad_w < 0)
     return I2CW_EINVAL;
   if (!vol && (D != 1 || T != 1 || pad_d != 0)) return I2CW_EINVAL;
+  if (prec != 0 && prec != 1) return I2CW_EINVAL;
+  if (prec && vol) return I2CW_EUNSUPPORTED;  // 1xTF32 kernels: 2D only
   Choice ch;
-  if (!choose(S, &ch)) return I2CW_EUNSUPPORTED;
-  // the 3D kernels are instantiated for the default alpha = 8 / 12 families only
-  if (vol && ch.alpha != 8 && ch.alpha != 12) ch = Choice{S <= 7 ? 9 - S : 13 - S, S <= 7 ? 8 : 12, 0};
+  if (!choose(S, C, &ch)) return I2CW_EUNSUPPORTED;
+  // the 3D and 1xTF32 kernels are instantiated for the default alpha = 8 / 12 families only
+  if ((vol || prec) && ch.alpha != 8 && ch.alpha != 12) ch = Choice{S <= 7 ? 9 - S : 13 - S, S <= 7 ? 8 : 12, 0};
   if (C % 4 != 0 || K % 4 != 0) return I2CW_EUNSUPPORTED;
   pl.N = N; pl.H = H; pl.W = W; pl.C = C; pl.K = K; pl.R = R; pl.S = S;
-  pl.vol = vol; pl.D = D; pl.T = T;
+  pl.vol = vol; pl.D = D; pl.T = T; pl.prec = prec;
   pl.is_deconv = is_deconv;
   if (is_deconv) {  // deconv(x, w, pad) == conv(x, rot180(w)^T, R-1-pad) (3D: rotate all three taps)
     pl.pad_d = T - 1 - pad_d;
@@ -206,7 +217,7 @@ int make_plan_uncached(int N, int D, int H, int W, int C, int K, int T, int R, i
   // (c256 +11%), -2..-18% otherwise (cfg2, r2-r7, c64, c128). I2CW_PAIR=1/0 forces it.
   static const int pair_env = [] { const char* e = getenv("I2CW_PAIR"); return e ? (e[0] == '1' ? 1 : 0) : -1; }();
   pl.pair = pair_env >= 0 ? pair_env : ((pl.NKS >= 128 || pl.NB >= 4) ? 1 : 0);
-  if (vol) pl.pair = 0;  // 3D kernels: single-CTA instantiations only
+  if (vol || prec) pl.pair = 0;  // 3D and 1xTF32 kernels: single-CTA instantiations only
   // DEBUG timing ablation (never set in production; results are wrong when non-zero)
   static const int ablate = [] { const char* e = getenv("I2CW_ABLATE"); return e ? atoi(e) : 0; }();
   pl.ablate = ablate;
@@ -331,20 +342,20 @@ int make_plan_uncached(int N, int D, int H, int W, int C, int K, int T, int R, i
 // Plans are pure functions of the call's dimensions (and the device's SM count): memoised,
 // so repeated calls skip the block-shape search and the lane permutation.
 int make_plan3(int N, int D, int H, int W, int C, int K, int T, int R, int S, int pad_d, int pad_h, int pad_w,
-               int is_deconv, int vol, Plan* out) {
-  struct Key { int v[16]; };
+               int is_deconv, int vol, Plan* out, int prec = 0) {
+  struct Key { int v[17]; };
   static std::mutex mu;
   static std::vector<std::pair<Key, Plan>> memo;
   int dev = 0;
   if (cudaGetDevice(&dev) != cudaSuccess) { cudaGetLastError(); dev = -1; }
-  const Key k{{N, D, H, W, C, K, T, R, S, pad_d, pad_h, pad_w, is_deconv, vol, dev, g_kchunk_max.load()}};
+  const Key k{{N, D, H, W, C, K, T, R, S, pad_d, pad_h, pad_w, is_deconv, vol, prec, dev, g_kchunk_max.load()}};
   {
     std::lock_guard<std::mutex> lk(mu);
     for (auto& e : memo)
       if (std::memcmp(e.first.v, k.v, sizeof(k.v)) == 0) { *out = e.second; return I2CW_OK; }
   }
   Plan pl;
-  const int rc = make_plan_uncached(N, D, H, W, C, K, T, R, S, pad_d, pad_h, pad_w, is_deconv, vol, &pl);
+  const int rc = make_plan_uncached(N, D, H, W, C, K, T, R, S, pad_d, pad_h, pad_w, is_deconv, vol, prec, &pl);
   if (rc != I2CW_OK) return rc;
   std::lock_guard<std::mutex> lk(mu);
   if (memo.size() >= 256) memo.erase(memo.begin());
@@ -518,9 +529,7 @@ std::vector<double> g_cached(const Plan& pl, int point_set) {
 }
 
 int transform_into(const Plan& pl, int is_deconv, const float* w, void* u, cudaStream_t stream) {
-  Choice ch;
-  choose(pl.S, &ch);
-  const std::vector<double> G = g_cached(pl, ch.point_set);
+  const std::vector<double> G = g_cached(pl, pl.alpha == 16 ? 1 : 0);  // alt alpha = 16 points (R7)
   const UTag tag = make_tag(pl, is_deconv);
   static_assert(sizeof(UTag) <= kUTagBytes, "tag");
   float* ud = reinterpret_cast<float*>(static_cast<uint8_t*>(u) + kUTagBytes);
@@ -667,7 +676,7 @@ const char* i2cw_status_string(int s) {
   }
 }
 
-int i2cw_version(void) { return 100; }
+int i2cw_version(void) { return 20000; }
 
 int i2cw_conv2d_nhwc(int N, int H, int W, int C, int K, int R, int S, int pad_h, int pad_w, const float* x,
                      const float* w, float* y, i2cw_stream_t stream) {
@@ -720,6 +729,19 @@ int i2cw_conv2d_nchw(int N, int C, int H, int W, int K, int R, int S, int pad_h,
 int i2cw_deconv2d_nchw(int N, int C, int H, int W, int K, int R, int S, int pad_h, int pad_w, const float* x,
                        const float* w, float* y, i2cw_stream_t stream) {
   return nchw_common(1, N, C, H, W, K, R, S, pad_h, pad_w, x, w, y, (cudaStream_t)stream);
+}
+
+int i2cw_conv2d_nhwc_prec(int precision, int is_deconv, int N, int H, int W, int C, int K, int R, int S, int pad_h,
+                          int pad_w, const float* x, const float* w, float* y, i2cw_stream_t stream) {
+  if (precision == I2CW_PREC_3XTF32)
+    return conv_common(is_deconv ? 1 : 0, N, H, W, C, K, R, S, pad_h, pad_w, x, w, y, (cudaStream_t)stream, false);
+  if (precision != I2CW_PREC_1XTF32 || (is_deconv != 0 && is_deconv != 1)) return I2CW_EINVAL;
+  if (!x || !w || !y) return I2CW_EINVAL;
+  if (!aligned16(x) || !aligned16(w) || !aligned16(y)) return I2CW_EINVAL;
+  Plan pl;
+  int rc = make_plan3(N, 1, H, W, C, K, 1, R, S, 0, pad_h, pad_w, is_deconv, 0, &pl, 1);
+  if (rc != I2CW_OK) return rc;
+  return conv_plan(pl, is_deconv, x, w, y, (cudaStream_t)stream, false, nullptr);
 }
 
 int i2cw_conv3d_ndhwc(int N, int D, int H, int W, int C, int K, int T, int R, int S, int pad_d, int pad_h, int pad_w,
@@ -863,9 +885,10 @@ int i2cw_conv2d_nhwc_host(int is_deconv, int N, int H, int W, int C, int K, int 
   return rc;
 }
 
-int i2cw_plan(int S, int* m, int* alpha, int* point_set) {
+int i2cw_plan(int S, int C, int* m, int* alpha, int* point_set) {
   Choice c;
-  if (!choose(S, &c)) return I2CW_EUNSUPPORTED;
+  if (C <= 0) return I2CW_EINVAL;
+  if (!choose(S, C, &c)) return I2CW_EUNSUPPORTED;
   if (m) *m = c.m;
   if (alpha) *alpha = c.alpha;
   if (point_set) *point_set = c.point_set;

@@ -44,6 +44,7 @@ struct Plan {
   int NKC, CPC;         // K-chunks (launches) of the K loop, channel chunks per K-chunk (bounded accumulation)
   int CC0, CC1;         // this launch's channel chunks [CC0, CC1) (set per K-chunk launch)
   int ACCUM;            // 1: every pass adds into y (a K-chunk after the first)
+  int prec;             // 0: 3xTF32 (default, fp32 accuracy); 1: 1xTF32 (looser tolerance, f4)
   int NUS;              // U ring super-slots (KPS k-steps of GP points each)
   int OSB;              // bytes of one output staging buffer = NI*ROWS*TS*16*4 (TMA store box, 16 channels)
   int OSTRIDE;          // OSB rounded up to 1024 (swizzled TMA boxes need 1024-byte alignment)
@@ -467,6 +468,13 @@ __device__ __forceinline__ void mma_commit(uint64_t* bar) {
 __device__ __forceinline__ void tmem_st_x4(uint32_t taddr, float a, float b, float c, float d) {
   asm volatile("tcgen05.st.sync.aligned.32x32b.x4.b32 [%0], {%1, %2, %3, %4};" ::"r"(taddr), "r"(__float_as_uint(a)),
                "r"(__float_as_uint(b)), "r"(__float_as_uint(c)), "r"(__float_as_uint(d))
+               : "memory");
+}
+__device__ __forceinline__ void tmem_st_x8(uint32_t taddr, const float (&v)[8]) {
+  asm volatile("tcgen05.st.sync.aligned.32x32b.x8.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};" ::"r"(taddr),
+               "r"(__float_as_uint(v[0])), "r"(__float_as_uint(v[1])), "r"(__float_as_uint(v[2])),
+               "r"(__float_as_uint(v[3])), "r"(__float_as_uint(v[4])), "r"(__float_as_uint(v[5])),
+               "r"(__float_as_uint(v[6])), "r"(__float_as_uint(v[7]))
                : "memory");
 }
 // 16 consecutive columns of this thread's lane

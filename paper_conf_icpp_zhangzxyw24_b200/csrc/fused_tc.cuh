@@ -168,7 +168,10 @@ struct TcCfg {
 // the K loop is a virtual chunk vc = cc * T + fd: channel chunk cc at depth tap fd, staged as one
 // input box at depth d0 - pad_d + fd. The NI slices a tile block stacks are consecutive OUTPUT
 // depths of one image (2D: consecutive images). Stage 2 (the 1D Winograd along W) is unchanged.
-template <int M, int RW, int NT, bool PAIR, bool VOL = false>
+// P1 = true: the 1xTF32 precision mode ("1xTF32 with looser tolerance"):
+// only the hi*hi product per point (one UMMA instead of three), V stored as its
+// round-to-nearest tf32 hi only; U still carries hi and lo, the lo images are not read.
+template <int M, int RW, int NT, bool PAIR, bool VOL = false, bool P1 = false>
 __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
     fused_tc_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__ CUtensorMap ymap,
                     const __grid_constant__ Plan pl, const float* __restrict__ u) {
@@ -262,7 +265,11 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
   const int CC0 = pl.CC0, NCCL = pl.CC1 - pl.CC0;
   const int NKS = NCCL * pl.R;
   const int NKSP = (NKS + KPS - 1) / KPS * KPS;   // k-steps per pass padded to whole super-stages
-  constexpr int PROD_WARP = NWG * 4, UPROD_WARP = NWG * 4 + 1, ISS_WARP0 = NWG * 4 + 2;
+#ifndef I2CW_ROLE_SWAP
+#define I2CW_ROLE_SWAP 0  // experiment: 1 = issuer warps on SMSPs 0/1, producers on 2/3
+#endif
+  constexpr int PROD_WARP = NWG * 4 + (I2CW_ROLE_SWAP ? NISS : 0), UPROD_WARP = PROD_WARP + 1,
+                ISS_WARP0 = NWG * 4 + (I2CW_ROLE_SWAP ? 0 : 2);
 
   if (threadIdx.x == 0) {
     // transform-warp arrivals are warp-elected (one lane after __syncwarp): 128 or 512
@@ -407,6 +414,17 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
 #pragma unroll
           for (int t = 0; t < GP; ++t) {
             if (ABL(256)) break;  // DEBUG timing ablation: no TMEM stores of V
+            if constexpr (P1) {  // 1xTF32: hi only (8 columns)
+              float v8[8];
+#pragma unroll
+              for (int cp = 0; cp < 4; ++cp) {
+                float2 hi, lo;
+                split_tf32x2(V[t][cp], hi, lo);
+                v8[2 * cp] = hi.x; v8[2 * cp + 1] = hi.y;
+              }
+              tmem_st_x8(vbase + t * 16, v8);
+              continue;
+            }
             float v16[16];
 #pragma unroll
             for (int cp = 0; cp < 4; ++cp) {
@@ -668,14 +686,15 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
               const uint64_t bk = bdesc0 + (uint64_t)((us * USBYTES + pos * UBYTES) >> 4);
               const uint32_t va = tbase + VCOL + (ss * KPS + pos) * GP * 16;
               // product order lo*hi, hi*lo, hi*hi (small terms first), points innermost
+              constexpr int PROD0 = P1 ? 2 : 0;  // 1xTF32: the hi*hi product only
 #pragma unroll
-              for (int prod = 0; prod < 3; ++prod) {
+              for (int prod = PROD0; prod < 3; ++prod) {
 #pragma unroll
                 for (int pi = 0; pi < PPI; ++pi) {
                   const int tl = iss * PPI + pi;
                   const uint32_t a = va + tl * 16 + (prod == 0 ? 8 : 0);
                   const uint64_t bd = bk + (uint64_t)(((tl * 2 + (prod == 1 ? 1 : 0)) * BROWS * 32) >> 4);
-                  const uint32_t acc = (kl > 0 || prod > 0) ? 1u : 0u;
+                  const uint32_t acc = (kl > 0 || prod > PROD0) ? 1u : 0u;
                   if constexpr (PAIR) mma2_tf32_ts_warp(tbase + tl * NT, a, bd, idesc, acc);
                   else mma_tf32_ts_warp(tbase + tl * NT, a, bd, idesc, acc);
                 }
@@ -748,11 +767,11 @@ inline int persistent_ctas(int units, int per) {
   return (units < slots ? units : slots) * per;
 }
 
-template <int M, int RW, int NT, bool PAIR, bool VOL = false>
+template <int M, int RW, int NT, bool PAIR, bool VOL = false, bool P1 = false>
 static cudaError_t launch_tc_t(const CUtensorMap& xmap, const CUtensorMap& ymap, const Plan& pl, const float* u,
                                cudaStream_t stream) {
   using Cfg = TcCfg<M, RW, NT, PAIR>;
-  auto kern = fused_tc_kernel<M, RW, NT, PAIR, VOL>;
+  auto kern = fused_tc_kernel<M, RW, NT, PAIR, VOL, P1>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, pl.smem_bytes);
   if (e != cudaSuccess) return e;
   if constexpr (PAIR) {

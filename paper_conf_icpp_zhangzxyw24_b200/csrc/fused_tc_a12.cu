@@ -13,6 +13,7 @@ cudaError_t launch_fused_tc_a12(const CUtensorMap& xmap, const CUtensorMap& ymap
 #define I2CW_TC(MM, RR)                                                                               \
   case RR * 1000 + MM * 10 + 1:                                                                      \
     if (pl.vol) return launch_tc_t<MM, RR, 64, false, true>(xmap, ymap, pl, u, stream);               \
+    if (pl.prec) return launch_tc_t<MM, RR, 64, false, false, true>(xmap, ymap, pl, u, stream);       \
     return pl.pair ? launch_tc_t<MM, RR, 64, true>(xmap, ymap, pl, u, stream)                       \
                    : launch_tc_t<MM, RR, 64, false>(xmap, ymap, pl, u, stream);                     \
   case RR * 1000 + MM * 10 + 2:                                                                      \
@@ -20,6 +21,7 @@ cudaError_t launch_fused_tc_a12(const CUtensorMap& xmap, const CUtensorMap& ymap
                    : launch_tc_t<MM, RR, 128, false>(xmap, ymap, pl, u, stream);                    \
   case RR * 1000 + MM * 10 + 0:                                                                      \
     if (pl.vol) return launch_tc_t<MM, RR, 32, false, true>(xmap, ymap, pl, u, stream);               \
+    if (pl.prec) return launch_tc_t<MM, RR, 32, false, false, true>(xmap, ymap, pl, u, stream);       \
     return pl.pair ? launch_tc_t<MM, RR, 32, true>(xmap, ymap, pl, u, stream)                       \
                    : launch_tc_t<MM, RR, 32, false>(xmap, ymap, pl, u, stream);
     I2CW_TC(5, 8) I2CW_TC(4, 9)

@@ -45,7 +45,7 @@ def test_alpha12_large_channels_every_element(kind, r, c, dist):
 def _residue_cases():
     cases = []
     for r in range(2, 10):
-        m = i2cw.plan(r)[0]
+        m = i2cw.plan(r, 8)[0]
         p = r // 2
         for kind in ("conv", "deconv"):
             for res in range(m):
@@ -60,7 +60,7 @@ def _residue_cases():
 def test_every_width_residue(kind, r, W, res):
     p = r // 2
     y, yr, b = run_case(kind, 1, 6, W, 8, 12, r, r, p, p)
-    assert y.shape[2] % i2cw.plan(r)[0] == res
+    assert y.shape[2] % i2cw.plan(r, 8)[0] == res
     assert_parity(y, yr, b)
 
 

@@ -63,8 +63,8 @@ def main():
              "|---|---|---|---|---|---|---|---|"]
     t0 = time.time()
     for r, lab, rows, paper in TABLE3:
-        m, a, _ = i2cw.plan(r)
         for (oh, oc), pm in zip(rows, paper):
+            m, a, _ = i2cw.plan(r, oc)
             N = 1 if oh * oh * oc * oc * r * r > 2e9 else 2
             mx, mr, pl = run("conv", N, oh, oh, oc, oc, r, 1.0, 2.0)
             lines.append(f"| {r} | {lab} | F({m},{r}) {a} | {N}x{oh}x{oh}x{oc} | {pl['NKC']} | {mx:.2e} | {mr:.2e} | {pm:.2e} |")

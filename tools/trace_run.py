@@ -58,7 +58,7 @@ for name in sys.argv[1:] or ["cfg2"]:
     print("epilogue d_full wait (before, after):", v(27).tolist(), " end:", v(28).tolist())
     # per k-step critical path sample: ks 8..15
     print("kg: CTA0 WG arrive | CTA1 WG arrive | CTA0 issuer ready | issued | committed   (ns)")
-    for kg in range(8, 16):
+    for kg in range(8, min(16, len(w16), len(w17), len(w18))):
         g = kg % nwg; i = kg // nwg
         a0 = v(8 + g, 0)[i] if i < len(v(8 + g, 0)) else None
         a1 = v(8 + g, 1)[i] if i < len(v(8 + g, 1)) else None
@@ -69,12 +69,12 @@ for name in sys.argv[1:] or ["cfg2"]:
     r29, r16, r17 = v(29, 1), v(16, 1), v(17, 1)
     if len(r29):
         print("relay (CTA1): kg: after st_full, after u_full, after remote arrive")
-        for kg in range(8, 12):
+        for kg in range(8, min(12, len(r29), len(r16), len(r17))):
             print("   ", kg, r29[kg], r16[kg], r17[kg])
     u30, u31 = v(30), v(31)
     if len(u30):
         print("U producer (CTA0): kg: before u_empty wait, issue time, issuer ready (u_full done)")
-        for kg in range(0, 16):
+        for kg in range(0, min(16, len(u30), len(u31))):
             print("   ", kg, u30[kg], u31[kg], w16[kg] if kg < len(w16) else None)
     if os.environ.get("TIMELINE"):
         lab = {0: "start", 4: "after-slot", 8: "arrive", 19: "in_full?", 23: "in_full!"}
@@ -103,3 +103,8 @@ for name in sys.argv[1:] or ["cfg2"]:
             nxt = e27[b + 4] if b + 4 < 512 and e27[b + 4] >= 0 else -1
             print(f"   {c:3d} t={e27[b]} compute+sts {e27[b+2]-e27[b]} fence+wait {e27[b+3]-e27[b+2]} bar {e27[b+1]-e27[b+3]} "
                   f"-> next {nxt-e27[b+1] if nxt>=0 else None}")
+    if os.environ.get("ISSUER"):
+        print("issuer0 per super-stage: before-wait, after-waits, after-issue, after-commit (cycles, relative)")
+        w29, w16, w17, w18 = v(29), v(16), v(17), v(18)
+        for j in range(10, min(40, len(w18))):
+            print(f"   ss{j}: {w29[j]} +{w16[j]-w29[j]} +{w17[j]-w16[j]} +{w18[j]-w17[j]}  next-before {w29[j+1]-w18[j] if j+1 < len(w29) else None}")
