@@ -180,6 +180,16 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
   constexpr int A = Cfg::A, GP = Cfg::GP, NS = Cfg::NS, NISS = Cfg::NISS, NWG = Cfg::NWG;
   constexpr int NPASS = Cfg::NPASS, VCOL = Cfg::VCOL, PPI = Cfg::PPI, BROWS = Cfg::BROWS;
   const int NIS = pl.NIS;  // input stages (runtime: fills the shared-memory budget)
+#ifndef I2CW_CSPLIT
+#define I2CW_CSPLIT 0  // experiment: 1 = two warpgroups per k-step, split by channel quads
+#endif
+  constexpr bool CS = I2CW_CSPLIT && NWG == 4 && !P1;
+#ifndef I2CW_UWAIT_WG
+#define I2CW_UWAIT_WG 0  // experiment: 1 = the transform warpgroups (not the issuer) wait for U
+#endif
+  // UW: each transform warpgroup checks its k-step's U super-slot (while it waits for its V slot
+  // anyway) before arriving; the issuer's one wait per super-stage then covers V and U
+  constexpr bool UW = I2CW_UWAIT_WG;
   constexpr uint32_t UBYTES = Cfg::UBYTES;
   const uint32_t rank = PAIR ? cluster_ctarank() : 0u;  // 0 = MMA leader
 
@@ -278,7 +288,7 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
     for (int i = 0; i < NSS; ++i) {
       // the 4 warps of each of the KPS warpgroups of this super-stage; a pair leader also counts
       // the peer's 4 x KPS warps, which arrive remotely (no relay thread on the V path)
-      mbar_init(&st_full[i], KPS * 4 * (PAIR && rank == 0 ? 2 : 1));
+      mbar_init(&st_full[i], KPS * 4 * (CS ? 2 : 1) * (PAIR && rank == 0 ? 2 : 1));
     }
     for (int i = 0; i < NSLOT; ++i) mbar_init(&st_empty[i], NISS);
     // pair leader's U slot: its own expect_tx arrive + the peer's "my half landed" arrive
@@ -305,6 +315,10 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
     if constexpr (kRegSplit) setmaxnreg_inc<104>();
     // ===================== transform + epilogue warpgroups =====================
     const int g = warp / 4;           // k-steps kg = g (mod NWG), V slots kg % NSLOT
+    // CS (channel split, I2CW_CSPLIT): warpgroups 2p and 2p+1 share the k-steps kg = p (mod 2),
+    // each transforming and storing one 4-channel quad (hs = g & 1) of every point: half the
+    // loads, math and TMEM stores per warpgroup per k-step, a shorter slot round trip.
+    const int kpar = CS ? (g >> 1) : g, hs = g & 1;
     const int l = threadIdx.x % 128;  // TMEM lane == tile slot
     const int row_l = pl.lane_row[l], tw_l = pl.lane_tw[l], in_l = pl.lane_in[l];
     const bool has_slot = row_l != 0xFF;
@@ -335,6 +349,12 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
       else mbar_arrive(d_empty);
     };
     auto wait_slot = [&](int kg) {  // this slot's previous k-step consumed (tcgen05.commit per k-step)
+      if constexpr (UW) {  // this k-step's U super-slot landed (both halves on a pair leader)
+        if (!PAIR || rank == 0) {
+          const int sg = kg / KPS;
+          mbar_wait_tc<PAIR>(&u_full[sg % pl.NUS], (sg / pl.NUS) & 1);
+        }
+      }
       const int use = kg / NSLOT;
       if (use > 0) mbar_wait_tc<PAIR>(&st_empty[kg & (NSLOT - 1)], (use - 1) & 1);
     };
@@ -356,12 +376,64 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
         mbar_wait(&in_full[ist], iph);
         trace_rec(pl.trace, 23 + g, PASS * pl.NCC + cc, l == 0);
         const uint8_t* stage = in_smem + (size_t)ist * 2 * inplane;  // [NI*HBOX][WBOX][8 ch], 32B-swizzled
-        for (int fh = (g - kb) & (NWG - 1); fh < pl.R; fh += NWG) {
+        for (int fh = CS ? ((kpar - kb) & 1) : ((g - kb) & (NWG - 1)); fh < pl.R; fh += CS ? 2 : NWG) {
           const int kg = kb + fh;
           trace_rec(pl.trace, 0 + g, kg / NWG, l == 0);
           // V for this k-step computed into registers BEFORE waiting for the V slot: the slot
           // round trip (MMA of the slot's previous k-step -> commit -> here) then covers only
           // the split + TMEM stores, not the shared-memory loads and the B^T math.
+          if constexpr (CS) {
+            float2 Vh[GP][2];  // point tl, channel pair p of this warpgroup's quad hs
+            {
+              const int x0 = (in_l + fh) * pl.WBOX + col0;
+              const uint8_t* xrow = stage + (size_t)x0 * 32;
+              float2 d[A][2];
+#pragma unroll
+              for (int j = 0; j < A; ++j) {
+                const int sw = ((x0 + j) & 4) << 2;  // 16 * bit2(xs)
+                const float4 v = *reinterpret_cast<const float4*>(xrow + j * 32 + (hs ? 16 - sw : sw));
+                d[j][0] = make_float2(v.x, v.y);
+                d[j][1] = make_float2(v.z, v.w);
+              }
+              static_for<GP / 2>([&](auto Q_) {
+                constexpr int idx0 = PASS * GP + 2 * (int)Q_;
+                constexpr int tl0 = 2 * (int)Q_;
+#pragma unroll
+                for (int p = 0; p < 2; ++p) {
+                  if constexpr (idx0 == 0) {
+                    Vh[tl0][p] = bt_dot2<T, 0, 1, 0>(d, p);
+                    Vh[tl0 + 1][p] = bt_dot2<T, A - 1, 1, 0>(d, p);
+                  } else {
+                    constexpr int pa = point_of(idx0, A);
+                    const float2 E = bt_dot2<T, pa, 2, 0>(d, p);
+                    const float2 O = bt_dot2<T, pa, 2, 1>(d, p);
+                    Vh[tl0][p] = __fadd2_rn(E, O);
+                    Vh[tl0 + 1][p] = __ffma2_rn(make_float2(-1.f, -1.f), O, E);
+                  }
+                }
+              });
+            }
+            wait_slot(kg);
+            tc_fence_after();
+            trace_rec(pl.trace, 4 + g, kg / NWG, l == 0);
+            const uint32_t vbase = vbase0 + (uint32_t)(kg & (NSLOT - 1)) * GP * 16 + 4 * hs;
+            // point tl: hi of this quad's 4 channels at columns 16 tl + 4 hs, lo at 16 tl + 8 + 4 hs
+#pragma unroll
+            for (int t = 0; t < GP; ++t) {
+              float2 h0, l0, h1, l1;
+              split_tf32x2(Vh[t][0], h0, l0);
+              split_tf32x2(Vh[t][1], h1, l1);
+              tmem_st_x4(vbase + t * 16, h0.x, h0.y, h1.x, h1.y);
+              tmem_st_x4(vbase + t * 16 + 8, l0.x, l0.y, l1.x, l1.y);
+            }
+            trace_rec(pl.trace, 12 + g, kg / NWG, l == 0);
+            tmem_wait_st();
+            tc_fence_before();
+            __syncwarp();
+            if (lane32 == 0) arrive_st_full((kg / KPS) % NSS);
+            trace_rec(pl.trace, 8 + g, kg / NWG, l == 0);
+            continue;
+          }
           float2 V[GP][4];  // point tl, channel pair cp (channels 2cp, 2cp+1 of the chunk)
           if (ABL(1)) {  // DEBUG timing ablation: V = 0 without loads or math
 #pragma unroll
@@ -450,7 +522,7 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
       // owning warpgroup still takes its turn so the super-stage's arrival count is met
       for (int kl = NKS; kl < NKSP; ++kl) {
         const int kg = kgp + kl;
-        if ((kg & (NWG - 1)) != g) continue;
+        if (CS ? ((kg & 1) != kpar) : ((kg & (NWG - 1)) != g)) continue;
         wait_slot(kg);
         tc_fence_before();
         __syncwarp();
@@ -664,10 +736,10 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
           trace_rec(pl.trace, 29, sgi, iss == 0 && lane32 == 0);
           if constexpr (PAIR) {  // both CTAs' V (peer arrivals are remote) and both U halves
             mbar_wait_cluster(&st_full[ss], sph);
-            mbar_wait_cluster(&u_full[us], uph);
+            if constexpr (!UW) mbar_wait_cluster(&u_full[us], uph);
           } else {
             mbar_wait(&st_full[ss], sph);
-            mbar_wait(&u_full[us], uph);
+            if constexpr (!UW) mbar_wait(&u_full[us], uph);
           }
           tc_fence_after();
           trace_rec(pl.trace, 16, sgi, iss == 0 && lane32 == 0);

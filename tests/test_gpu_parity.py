@@ -137,3 +137,42 @@ def test_accuracy_band_paper_table3():
         assert_parity(y, yr, b)
         rel = np.abs(y.cpu().double().numpy() - yr) / np.abs(yr)
         assert rel.mean() < tol_mean, rel.mean()
+
+
+def test_two_threads_concurrent_shapes():
+    """Two host threads, each on its own CUDA stream, alternating different filter widths (the
+    plan memo, the G-table memo and the U tag registry are shared): every result equals the one
+    the same call produces alone, bit for bit."""
+    import threading
+    cases = [("conv", 2, 12, 29, 16, 24, r, r, r // 2, r // 2) for r in (2, 3, 5, 8)] + \
+            [("deconv", 2, 11, 23, 8, 40, r, r, r // 2, r // 2) for r in (4, 7, 9)]
+    data = [inputs(c[0], *c[1:8]) for c in cases]
+    ref = []
+    for c, (x, w) in zip(cases, data):
+        f = i2cw.conv2d_nhwc if c[0] == "conv" else i2cw.deconv2d_nhwc
+        ref.append(f(x.cuda(), w.cuda(), c[8], c[9]))
+    torch.cuda.synchronize()
+    out, errs = {}, []
+
+    def work(tid, order):
+        try:
+            s = torch.cuda.Stream()
+            with torch.cuda.stream(s):
+                for rep in range(3):
+                    for i in order:
+                        c, (x, w) = cases[i], data[i]
+                        f = i2cw.conv2d_nhwc if c[0] == "conv" else i2cw.deconv2d_nhwc
+                        out[(tid, rep, i)] = f(x.cuda(), w.cuda(), c[8], c[9], stream=s)
+            s.synchronize()
+        except Exception as e:  # pragma: no cover - reported below
+            errs.append(e)
+
+    ts = [threading.Thread(target=work, args=(0, list(range(len(cases))))),
+          threading.Thread(target=work, args=(1, list(reversed(range(len(cases))))))]
+    for t in ts:
+        t.start()
+    for t in ts:
+        t.join()
+    assert not errs, errs
+    for (tid, rep, i), y in out.items():
+        assert torch.equal(y, ref[i]), (tid, rep, cases[i])

@@ -1,6 +1,6 @@
-"""Summarise an ncu --set full capture of the fused kernel (run here, no GPU needed):
-  python tools/ncu_summary.py gpurun_out/prof_X.ncu-rep CONFIG_NAME > profiles/..._summary.md
-Also merges the kernel's DRAM traffic per launch into profiles/traffic.json."""
+"""Summarise an ncu --set full capture of the fused kernel (no GPU needed):
+  python tools/ncu_summary.py gpurun_out/prof_X.ncu-rep CONFIG_NAME [traffic.json] > ..._summary.md
+Also merges the kernel's DRAM traffic per launch into traffic.json (default profiles/traffic.json)."""
 import csv, io, json, os, subprocess, sys
 
 rep, cfg = sys.argv[1], sys.argv[2]
@@ -15,7 +15,11 @@ keys = ["Kernel Name", "gpu__time_duration.sum", "launch__grid_size", "launch__b
         "lts__throughput.avg.pct_of_peak_sustained_elapsed",
         "l1tex__data_pipe_lsu_wavefronts_mem_shared_op_ld.sum", "l1tex__data_bank_conflicts_pipe_lsu_mem_shared_op_ld.sum",
         "l1tex__data_pipe_lsu_wavefronts_mem_shared_op_st.sum", "l1tex__data_bank_conflicts_pipe_lsu_mem_shared_op_st.sum",
-        "sm__warps_active.avg.pct_of_peak_sustained_active"]
+        "sm__warps_active.avg.pct_of_peak_sustained_active",
+        "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum.pct_of_peak_sustained_elapsed",
+        "l1tex__data_pipe_tc_wavefronts_mem_shared.sum.pct_of_peak_sustained_elapsed",
+        "l1tex__m_xbar2l1tex_read_bytes.sum.pct_of_peak_sustained_elapsed",
+        "lts__t_sectors_srcunit_tex_op_red.sum"]
 print(f"# ncu --set full summary: {cfg} ({os.path.basename(rep)})\n")
 print("| metric | value | unit |\n|---|---|---|")
 for k in keys:
@@ -32,7 +36,8 @@ for k, v in stalls[:8]:
 rd, _ = get("dram__bytes_read.sum"); wr, u = get("dram__bytes_write.sum")
 scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}.get(u, 1)
 traffic = (float(rd) + float(wr)) * scale
-path = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "profiles", "traffic.json")
+path = sys.argv[3] if len(sys.argv) > 3 else os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))),
+                                                         "profiles", "traffic.json")
 d = json.load(open(path)) if os.path.exists(path) else {}
 d[cfg] = traffic
 json.dump(d, open(path, "w"), indent=1, sort_keys=True)
