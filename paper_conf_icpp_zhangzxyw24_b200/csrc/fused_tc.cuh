@@ -570,7 +570,14 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
             }
           }
         });
-        if (l == 0) bulk_wait_group_read_dyn(pl.NOB - 1);  // buffer 0: previous pass's stores
+        if (l == 0) {
+          bulk_wait_group_read_dyn(pl.NOB - 1);  // buffer 0: previous pass's stores
+          // a later pass of the same unit reduce-adds onto what the previous pass wrote: those
+          // writes must be complete (bulk operations are not ordered with each other). Waited
+          // here, a whole mainloop after they were issued, instead of at the end of that pass
+          // where the wait sat on the next pass's first V (thread 0 is in warp 0 of the group)
+          if (PASS > 0 && !I.split) bulk_wait_group_all();
+        }
         named_bar_sync(1 + g, 128);
         trace_rec(pl.trace, 28, 129 + 2 * gpass, l == 0 && g == 0);
         static_for<M>([&](auto I_) {
@@ -632,8 +639,8 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
           }
         });
       }
-      // this pass's writes must be complete before the next pass's reduce-add
-      if (l == 0) bulk_wait_group_all();
+      // staging buffers free for the next pass (its writes complete later, see above)
+      if (l == 0) bulk_wait_group_read<0>();
       trace_rec(pl.trace, 28, gpass, l == 0 && g == 0);
     });
     }  // units
