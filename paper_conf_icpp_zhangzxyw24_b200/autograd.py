@@ -11,7 +11,7 @@ from __future__ import annotations
 
 import torch
 
-from . import conv2d_nhwc, deconv2d_nhwc
+from . import conv2d_nhwc, conv3d_ndhwc, deconv2d_nhwc, deconv3d_ndhwc
 
 
 class Conv2dNHWC(torch.autograd.Function):
@@ -39,3 +39,29 @@ class Conv2dNHWC(torch.autograd.Function):
 def conv2d(x: torch.Tensor, w: torch.Tensor, pad_h: int, pad_w: int) -> torch.Tensor:
     """Differentiable (w.r.t. x) fused Im2col-Winograd convolution, NHWC x, KRSC w."""
     return Conv2dNHWC.apply(x, w, pad_h, pad_w)
+
+
+class Conv3dNDHWC(torch.autograd.Function):
+    """3D (PAPER.md:314-315): y = conv3d(x, w, pad) in NDHWC / KTRSC; grad_x = deconv3d(grad_y, w, pad)."""
+
+    @staticmethod
+    def forward(ctx, x, w, pad_d: int, pad_h: int, pad_w: int):
+        ctx.save_for_backward(w)
+        ctx.pad = (pad_d, pad_h, pad_w)
+        return conv3d_ndhwc(x.contiguous(), w.contiguous(), pad_d, pad_h, pad_w)
+
+    @staticmethod
+    def backward(ctx, grad_y):
+        (w,) = ctx.saved_tensors
+        if ctx.needs_input_grad[1]:
+            raise NotImplementedError("i2cw: backward-filter (dW) is outside Im2col-Winograd; "
+                                      "detach the filter or compute dW elsewhere")
+        grad_x = None
+        if ctx.needs_input_grad[0]:
+            grad_x = deconv3d_ndhwc(grad_y.contiguous(), w, *ctx.pad)
+        return grad_x, None, None, None, None
+
+
+def conv3d(x: torch.Tensor, w: torch.Tensor, pad_d: int, pad_h: int, pad_w: int) -> torch.Tensor:
+    """Differentiable (w.r.t. x) 3D fused Im2col-Winograd convolution, NDHWC x, KTRSC w."""
+    return Conv3dNDHWC.apply(x, w, pad_d, pad_h, pad_w)

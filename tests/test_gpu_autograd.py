@@ -7,7 +7,7 @@ import pytest
 import torch
 
 import oracle
-from paper_conf_icpp_zhangzxyw24_b200.autograd import conv2d
+from paper_conf_icpp_zhangzxyw24_b200.autograd import conv2d, conv3d
 from synthetic import make_w, make_x
 
 pytestmark = pytest.mark.gpu
@@ -34,3 +34,17 @@ def test_filter_gradient_not_offered():
     y = conv2d(x, w, 1, 1)
     with pytest.raises(NotImplementedError):
         y.sum().backward()
+
+
+def test_backward_data_3d_matches_oracle():
+    g = torch.Generator().manual_seed(5)
+    x = (torch.rand((2, 6, 9, 13, 16), generator=g) * 2 - 1).cuda().requires_grad_(True)
+    w = (torch.rand((24, 3, 3, 5, 16), generator=g) * 2 - 1).cuda()
+    y = conv3d(x, w, 1, 1, 2)
+    dy = torch.rand(y.shape, generator=g) * 2 - 1
+    y.backward(dy.cuda())
+    torch.cuda.synchronize()
+    ref, bound = oracle.deconv3d_ndhwc(dy, w.cpu(), 1, 1, 2)
+    got = x.grad.double().cpu().numpy()
+    assert got.shape == ref.shape
+    assert float(np.max(np.abs(got - ref) / np.maximum(bound, 1e-30))) <= 1e-4

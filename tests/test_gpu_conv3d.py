@@ -74,3 +74,9 @@ def test_conv3d_deterministic_and_2d_equivalence():
     _, b = oracle.conv2d_nhwc(x[:, 0], w[:, 0], 1, 2)
     r = float(((y1[:, 0] - y2d).abs().double().cpu() / torch.as_tensor(b).clamp_min(1e-30)).max())
     assert r <= 2e-4
+
+
+def test_conv3d_video_layer_full_check():
+    """A video-style 3x3x3 layer (N=2, 8 frames of 28x28, C=K=64): every output element."""
+    y, yr, b = run3("conv", 2, 8, 28, 28, 64, 64, 3, 3, 3, 1, 1, 1, seed=21)
+    assert_parity(y, yr, b)
