@@ -28,6 +28,8 @@ def max_over_ranks(values, device=None) -> list[float]:
     """Element-wise MAX of a list of floats over all ranks (identity without a process group)."""
     t = torch.tensor([float(v) for v in values], dtype=torch.float64, device=device)
     if dist.is_available() and dist.is_initialized() and dist.get_world_size() > 1:
+        if dist.get_backend() == "gloo":  # gloo collectives on host tensors
+            t = t.cpu()
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     return t.tolist()
 
@@ -37,6 +39,8 @@ def gather_rows(local: torch.Tensor) -> torch.Tensor:
     largest, then trimmed); returns the concatenation in rank order on every rank."""
     if not (dist.is_available() and dist.is_initialized()) or dist.get_world_size() == 1:
         return local
+    if dist.get_backend() == "gloo" and local.is_cuda:  # gloo collectives on host tensors
+        return gather_rows(local.cpu()).to(local.device)
     world = dist.get_world_size()
     n = torch.tensor([local.shape[0]], dtype=torch.int64, device=local.device)
     ns = [torch.zeros_like(n) for _ in range(world)]
