@@ -429,7 +429,9 @@ def main():
                      "ms": t_star / args.steps * 1e3,
                      "what": "pre-transformed filter (the paper's '*', PAPER.md:3951-3952): fused kernel only"},
             # one-shot call = filter transform + one fused launch per K-chunk (+ split-tail zeroing)
-            "gpu_launches": (1 + p["NKC"] + (1 if p["NITEMS"] != p["NFULL"] else 0)) * args.steps,
+            # filter transform + per K slice (K-chunk launches + split-tail zeroing) + slice combine
+            "gpu_launches": (1 + p["KSL"] * (p["NKC"] + (1 if p["NITEMS"] != p["NFULL"] else 0))
+                             + (1 if p["KSL"] > 1 else 0)) * args.steps,
             "outputs_finite": ok_all,
             "clocks": clocks,
         }

@@ -27,13 +27,21 @@
  *    stream-ordered workspace pool (see i2cw_conv2d_nhwc), a memo of launch plans
  *    and transform tables (pure functions of the dimensions), and two copy streams
  *    per device for i2cw_conv2d_nhwc_host.
- *  - A conv/deconv call may enqueue a small zeroing kernel on part of y before its
- *    fused kernel (the "split tail" of the persistent schedule, whose two Winograd
- *    passes both reduce-add into y); it is a programmatic dependent of the previous
- *    kernel in the stream and writes only y. Results are bitwise deterministic.
+ *  - A conv/deconv call enqueues the filter transform, then one fused launch per
+ *    K-chunk (a K loop longer than 256 k-steps for alpha <= 8 / 128 for alpha = 12,
+ *    one k-step = 8 channels x 1 filter row, runs as several launches whose partial
+ *    sums are added into y in order: the tcgen05 fp32 accumulator truncates once per
+ *    MMA, so bounding the accumulation length bounds the error for any C), and may
+ *    enqueue a small zeroing kernel on part of y before the first fused launch (the
+ *    "split tail" of the persistent schedule, whose two Winograd passes both
+ *    reduce-add into y). The zeroing kernel is a programmatic dependent of the
+ *    previous kernel and touches y only after that kernel's grid has completed unless
+ *    that kernel is the library's own filter transform. Results are bitwise
+ *    deterministic run to run.
  *  - fp32 in / fp32 out. The per-point channel contraction runs on the tcgen05
- *    tensor cores in 3xTF32 (hi*hi + hi*lo + lo*hi), which keeps
- *    |y - y_exact| <= 1e-4 * sum|x|*|w| per element (BASELINE.json north_star).
+ *    tensor cores in 3xTF32 (hi*hi + hi*lo + lo*hi, V split to nearest tf32), which
+ *    keeps |y - y_exact| <= 1e-4 * sum|x|*|w| per element (BASELINE.json north_star);
+ *    i2cw_conv2d_nhwc_prec offers a 1xTF32 mode with a looser stated bound.
  *  - No CPU fallback: on a machine without a B200 the calls return I2CW_ECUDA.
  *
  * Return codes (i2cw_status): 0 on success, negative on error; nothing is
@@ -42,7 +50,7 @@
  *                     misaligned pointer, tag mismatch on a pre-transformed filter.
  *   I2CW_EUNSUPPORTED S outside [2, 9]; C % 4 != 0 or K % 4 != 0 (TMA global strides
  *                     and 16-byte vector stores need 16-byte rows); a shape whose
- *                     tile plan exceeds the on-chip budget.
+ *                     tile plan exceeds the on-chip budget or a TMA box limit.
  *   I2CW_ECUDA        a CUDA runtime error (no device, launch failure, OOM).
  */
 #ifndef I2CW_H_

@@ -86,6 +86,9 @@ def lib():
         if hasattr(L, "i2cw_debug_set_kchunk"):  # test hook (absent from older experiment builds)
             L.i2cw_debug_set_kchunk.argtypes = [I]
             L.i2cw_debug_set_kchunk.restype = I
+        if hasattr(L, "i2cw_debug_set_kslices"):
+            L.i2cw_debug_set_kslices.argtypes = [I]
+            L.i2cw_debug_set_kslices.restype = I
         _lib = L
     return _lib
 
@@ -99,10 +102,14 @@ def _check(fn, rc):
         raise I2CWError(fn, rc)
 
 
-def _stream_ptr(stream):
+def _stream_ptr(stream, like=None):
+    """The raw cudaStream_t: the given torch stream, else the current stream of like's device
+    (the device the library binds for the call), else of the current device."""
+    if stream is not None:
+        return stream.cuda_stream
     import torch
-    s = stream if stream is not None else torch.cuda.current_stream()
-    return s.cuda_stream
+    dev = like.get_device() if like is not None else torch.cuda.current_device()
+    return torch._C._cuda_getCurrentRawStream(dev)
 
 
 def _check_tensor(t, name):
@@ -143,10 +150,10 @@ def conv2d_nhwc(x, w, pad_h, pad_w, out=None, stream=None, precision="3xtf32"):
     if precision != "3xtf32":
         _check("i2cw_conv2d_nhwc_prec", lib().i2cw_conv2d_nhwc_prec(
             PRECISIONS[precision], 0, N, H, W, C, K, R, S, pad_h, pad_w, x.data_ptr(), w.data_ptr(), y.data_ptr(),
-            _stream_ptr(stream)))
+            _stream_ptr(stream, x)))
         return y
     _check("i2cw_conv2d_nhwc", lib().i2cw_conv2d_nhwc(N, H, W, C, K, R, S, pad_h, pad_w, x.data_ptr(), w.data_ptr(),
-                                                      y.data_ptr(), _stream_ptr(stream)))
+                                                      y.data_ptr(), _stream_ptr(stream, x)))
     return y
 
 
@@ -163,10 +170,10 @@ def deconv2d_nhwc(x, w, pad_h, pad_w, out=None, stream=None, precision="3xtf32")
     if precision != "3xtf32":
         _check("i2cw_conv2d_nhwc_prec", lib().i2cw_conv2d_nhwc_prec(
             PRECISIONS[precision], 1, N, H, W, C, K, R, S, pad_h, pad_w, x.data_ptr(), w.data_ptr(), y.data_ptr(),
-            _stream_ptr(stream)))
+            _stream_ptr(stream, x)))
         return y
     _check("i2cw_deconv2d_nhwc", lib().i2cw_deconv2d_nhwc(N, H, W, C, K, R, S, pad_h, pad_w, x.data_ptr(),
-                                                          w.data_ptr(), y.data_ptr(), _stream_ptr(stream)))
+                                                          w.data_ptr(), y.data_ptr(), _stream_ptr(stream, x)))
     return y
 
 
@@ -180,7 +187,7 @@ def conv2d_nchw(x, w, pad_h, pad_w, out=None, stream=None):
     _, P, Q, _ = out_shape("conv", N, H, W, K, R, S, pad_h, pad_w)
     y = _out(out, (N, K, P, Q), x)
     _check("i2cw_conv2d_nchw", lib().i2cw_conv2d_nchw(N, C, H, W, K, R, S, pad_h, pad_w, x.data_ptr(), w.data_ptr(),
-                                                      y.data_ptr(), _stream_ptr(stream)))
+                                                      y.data_ptr(), _stream_ptr(stream, x)))
     return y
 
 
@@ -194,7 +201,7 @@ def deconv2d_nchw(x, w, pad_h, pad_w, out=None, stream=None):
     _, P, Q, _ = out_shape("deconv", N, H, W, K, R, S, pad_h, pad_w)
     y = _out(out, (N, K, P, Q), x)
     _check("i2cw_deconv2d_nchw", lib().i2cw_deconv2d_nchw(N, C, H, W, K, R, S, pad_h, pad_w, x.data_ptr(),
-                                                          w.data_ptr(), y.data_ptr(), _stream_ptr(stream)))
+                                                          w.data_ptr(), y.data_ptr(), _stream_ptr(stream, x)))
     return y
 
 
@@ -213,7 +220,7 @@ def conv3d_ndhwc(x, w, pad_d, pad_h, pad_w, out=None, stream=None):
         raise ValueError("channel or device mismatch")
     y = _out(out, out_shape3("conv", N, D, H, W, K, T, R, S, pad_d, pad_h, pad_w), x)
     _check("i2cw_conv3d_ndhwc", lib().i2cw_conv3d_ndhwc(N, D, H, W, C, K, T, R, S, pad_d, pad_h, pad_w, x.data_ptr(),
-                                                        w.data_ptr(), y.data_ptr(), _stream_ptr(stream)))
+                                                        w.data_ptr(), y.data_ptr(), _stream_ptr(stream, x)))
     return y
 
 
@@ -227,7 +234,7 @@ def deconv3d_ndhwc(x, w, pad_d, pad_h, pad_w, out=None, stream=None):
     y = _out(out, out_shape3("deconv", N, D, H, W, K, T, R, S, pad_d, pad_h, pad_w), x)
     _check("i2cw_deconv3d_ndhwc", lib().i2cw_deconv3d_ndhwc(N, D, H, W, C, K, T, R, S, pad_d, pad_h, pad_w,
                                                             x.data_ptr(), w.data_ptr(), y.data_ptr(),
-                                                            _stream_ptr(stream)))
+                                                            _stream_ptr(stream, x)))
     return y
 
 
@@ -249,7 +256,7 @@ def filter_transform(w, is_deconv=False, stream=None):
         raise I2CWError("i2cw_filter_bytes", I2CW_EUNSUPPORTED)
     u = torch.empty(nbytes, dtype=torch.uint8, device=w.device)
     _check("i2cw_filter_transform", lib().i2cw_filter_transform(K, C, R, S, int(bool(is_deconv)), w.data_ptr(),
-                                                                u.data_ptr(), _stream_ptr(stream)))
+                                                                u.data_ptr(), _stream_ptr(stream, w)))
     return u
 
 
@@ -267,7 +274,7 @@ def conv2d_nhwc_pretransformed(x, u, K, R, S, pad_h, pad_w, is_deconv=False, out
     y = _out(out, out_shape("deconv" if is_deconv else "conv", N, H, W, K, R, S, pad_h, pad_w), x)
     fn = lib().i2cw_deconv2d_nhwc_pretransformed if is_deconv else lib().i2cw_conv2d_nhwc_pretransformed
     _check("i2cw_*_pretransformed", fn(N, H, W, C, K, R, S, pad_h, pad_w, x.data_ptr(), u.data_ptr(), y.data_ptr(),
-                                       _stream_ptr(stream)))
+                                       _stream_ptr(stream, x)))
     return y
 
 
@@ -321,7 +328,7 @@ def transform_matrices(m, r, point_set=0):
 
 PLAN_FIELDS = ("P", "Q", "m", "alpha", "NT", "NB", "NCC", "NKS", "T_r", "TS", "SEGS", "ROWS", "PB", "WBOX", "HBOX",
                "tile_blocks", "GP", "NPASS", "NUS", "smem_bytes", "pad_h", "pad_w", "NI", "NFULL", "NITEMS", "pair",
-               "NKC", "CPC")
+               "NKC", "CPC", "KSL")
 
 
 def debug_plan(kind, N, H, W, C, K, R, S, pad_h, pad_w):
@@ -337,6 +344,12 @@ def debug_set_kchunk(ksteps: int) -> int:
     return int(lib().i2cw_debug_set_kchunk(int(ksteps)))
 
 
+def debug_set_kslices(n: int) -> int:
+    """TEST-ONLY: cap on concurrent K slices for small grids (1 disables, 0 = default 4);
+    returns the old setting (-1 = default)."""
+    return int(lib().i2cw_debug_set_kslices(int(n)))
+
+
 def debug_conv_simt(x, w, pad_h, pad_w, is_deconv=False, stream=None):
     """TEST-ONLY: the SIMT stepping-stone kernel on the same plan / U (not the product path)."""
     import torch
@@ -350,5 +363,5 @@ def debug_conv_simt(x, w, pad_h, pad_w, is_deconv=False, stream=None):
     y = torch.empty(shp, dtype=torch.float32, device=x.device)
     _check("i2cw_debug_conv_simt", lib().i2cw_debug_conv_simt(int(bool(is_deconv)), N, H, W, C, K, R, S, pad_h,
                                                               pad_w, x.data_ptr(), w.data_ptr(), y.data_ptr(),
-                                                              _stream_ptr(stream)))
+                                                              _stream_ptr(stream, x)))
     return y

@@ -25,6 +25,7 @@ cudaError_t launch_fused_tc(const CUtensorMap& xmap, const CUtensorMap& ymap, co
                             cudaStream_t stream);
 cudaError_t launch_zero_tail(float* y, size_t count, bool wait_first, cudaStream_t stream);
 cudaError_t launch_transpose(const float* in, float* out, int B, int rows, int cols, cudaStream_t stream);
+cudaError_t launch_ksum(float* y, const float* slices, int nslices, size_t count, size_t stride, cudaStream_t stream);
 cudaError_t launch_fused_simt(const Plan& pl, const float* x, const float* u, float* y, cudaStream_t stream);
 
 namespace {
@@ -43,6 +44,14 @@ constexpr int kSmemBudget = 225 * 1024;
 // i2cw_debug_set_kchunk (test hook) overrides the cap so small parity cases exercise chunking.
 int kchunk_default(int alpha) { return alpha <= 8 ? 256 : (alpha <= 12 ? 128 : 64); }
 std::atomic<int> g_kchunk_max{0};  // 0: kchunk_default(alpha)
+// Cap on concurrent K slices for small grids (run_fused); -1: default (4, or I2CW_KSLICES).
+std::atomic<int> g_kslices_max{-1};
+constexpr int kMaxKSlices = 8;
+int kslices_cap() {
+  static const int env = [] { const char* e = getenv("I2CW_KSLICES"); return e ? std::max(1, atoi(e)) : 4; }();
+  const int v = g_kslices_max.load();
+  return std::min(kMaxKSlices, v > 0 ? v : env);
+}
 
 // Per filter width S: F(m, S) and the point set. r = 2..7 follow the paper's
 // Gamma_8 choices (Table 2). For r = 8, 9 the paper uses
@@ -335,6 +344,18 @@ int make_plan_uncached(int N, int D, int H, int W, int C, int K, int T, int R, i
       pl.NFULL = pl.NITEMS = units;
     }
   }
+  // K slices (run_fused): when the work items fill at most half of the SMs and the K loop is
+  // one chunk, up to kslices_cap() slices of the channel chunks run concurrently, each item
+  // keeping >= 64 k-step passes (shorter slices save less device time than the extra launches
+  // cost on the host: measured on B200, profiles/r02_kslice_ab.txt)
+  {
+    const int ctas = pl.pair ? 2 * pl.NITEMS : pl.NITEMS;
+    const int item_ksteps = pl.NKS * (pl.NFULL > 0 ? pl.NPASS : 1);
+    pl.KSL = 1;
+    if (pl.NKC == 1 && pl.NCC >= 2 && 2 * ctas <= nsm)
+      pl.KSL = std::max(1, std::min({kslices_cap(), pl.NCC, nsm / std::max(1, ctas), item_ksteps / 64}));
+    if (pl.KSL > 1) pl.KSL = cdiv(pl.NCC, cdiv(pl.NCC, pl.KSL));  // no empty slice
+  }
   *out = pl;
   return I2CW_OK;
 }
@@ -343,12 +364,12 @@ int make_plan_uncached(int N, int D, int H, int W, int C, int K, int T, int R, i
 // so repeated calls skip the block-shape search and the lane permutation.
 int make_plan3(int N, int D, int H, int W, int C, int K, int T, int R, int S, int pad_d, int pad_h, int pad_w,
                int is_deconv, int vol, Plan* out, int prec = 0) {
-  struct Key { int v[17]; };
+  struct Key { int v[18]; };
   static std::mutex mu;
   static std::vector<std::pair<Key, Plan>> memo;
   int dev = 0;
   if (cudaGetDevice(&dev) != cudaSuccess) { cudaGetLastError(); dev = -1; }
-  const Key k{{N, D, H, W, C, K, T, R, S, pad_d, pad_h, pad_w, is_deconv, vol, prec, dev, g_kchunk_max.load()}};
+  const Key k{{N, D, H, W, C, K, T, R, S, pad_d, pad_h, pad_w, is_deconv, vol, prec, dev, g_kchunk_max.load(), kslices_cap()}};
   {
     std::lock_guard<std::mutex> lk(mu);
     for (auto& e : memo)
@@ -545,7 +566,16 @@ int transform_into(const Plan& pl, int is_deconv, const float* w, void* u, cudaS
 // never touches y), so the zeroing kernel may overlap it through programmatic dependent launch;
 // otherwise (pre-transformed path: the caller's last kernel is unknown) the zeroing kernel
 // waits for the previous grid before its first store.
-int run_fused(const Plan& pl, const float* x, const void* u, float* y, bool after_own_ft, cudaStream_t stream) {
+// A failed CUDA call on the launch path: clears the error, logs it with I2CW_VERBOSE=1.
+int cuda_fail(const char* what) {
+  static const bool verbose = [] { const char* e = getenv("I2CW_VERBOSE"); return e && e[0] == '1'; }();
+  const cudaError_t e = cudaGetLastError();
+  if (verbose) fprintf(stderr, "i2cw: %s failed: %s\n", what, cudaGetErrorString(e));
+  return I2CW_ECUDA;
+}
+
+// One fused launch sequence (K-chunks in order, split-tail zeroing first) writing y.
+int run_fused_into(const Plan& pl, const float* x, const void* u, float* y, bool after_own_ft, cudaStream_t stream) {
   CUtensorMap map, ymap;
   if (pl.NITEMS != pl.NFULL) {
     // split tail: both passes of a tail unit reduce-add into y, so y is zeroed from the first
@@ -556,7 +586,7 @@ int run_fused(const Plan& pl, const float* x, const void* u, float* y, bool afte
     const size_t img = (size_t)pl.OD * pl.P * pl.Q * pl.K;
     if (n0 < (size_t)pl.N &&
         launch_zero_tail(y + n0 * img, ((size_t)pl.N - n0) * img, !after_own_ft, stream) != cudaSuccess)
-      return I2CW_ECUDA;
+      return cuda_fail("zero tail");
   }
   int rc = encode_x_map(pl, x, &map);
   if (rc != I2CW_OK) return rc;
@@ -564,18 +594,80 @@ int run_fused(const Plan& pl, const float* x, const void* u, float* y, bool afte
   const float* ud = reinterpret_cast<const float*>(static_cast<const uint8_t*>(u) + kUTagBytes);
   // K-chunks: one launch per chunk of <= CPC channel chunks, in order on the
   // stream; the first stores y (its split tail reduce-adds into the zeroed region), later ones
-  // reduce-add every pass. Sequential launches keep the fp32 summation order fixed.
+  // add every pass. Sequential launches keep the fp32 summation order fixed.
   for (int kc = 0; kc < pl.NKC; ++kc) {
     Plan pk = pl;
-    pk.CC0 = kc * pl.CPC;
-    pk.CC1 = std::min(pl.NCC, pk.CC0 + pl.CPC);
+    pk.CC0 = pl.CC0 + kc * pl.CPC;
+    pk.CC1 = std::min(pl.CC1, pk.CC0 + pl.CPC);
     pk.ACCUM = kc > 0;
     // the split tail's two one-pass items per unit add in either order: exact only onto y = 0
     // (0 + a + b), so later chunks (y != 0) run every unit whole, its passes in order
     if (kc > 0) pk.NFULL = pk.NITEMS = pl.NFULL + (pl.NITEMS - pl.NFULL) / 2;
-    if (launch_fused_tc(map, ymap, pk, ud, stream) != cudaSuccess) return I2CW_ECUDA;
+    if (launch_fused_tc(map, ymap, pk, ud, stream) != cudaSuccess) return cuda_fail("fused launch");
   }
   return I2CW_OK;
+}
+
+// Small grids (SURVEY.md §7 hard part 7, §8(e): a per-GPU shard of a few images leaves most
+// SMs idle, and one work unit's latency sets the time): the K loop is split into S slices
+// launched CONCURRENTLY on forked streams, each into its own y-sized workspace (slice 0 into
+// y), and a combine kernel sums the slices in a fixed order -- deterministic, and each slice's
+// accumulation is shorter (more accurate). The planner sets S = Plan::KSL (make_plan_uncached).
+// Per-device fork/join resources, created once: the slice streams and events. The mutex is
+// held while a call issues its fork/join (host side, a few microseconds), so concurrent host
+// threads never interleave records of the shared events.
+struct ForkCtx {
+  std::mutex mu;
+  bool ready = false;
+  cudaStream_t st[kMaxKSlices - 1] = {};
+  cudaEvent_t ev[kMaxKSlices] = {};
+};
+
+ForkCtx* fork_ctx(int dev) {
+  static ForkCtx ctx[64];
+  return dev >= 0 && dev < 64 ? &ctx[dev] : nullptr;
+}
+
+int run_fused(const Plan& pl, const float* x, const void* u, float* y, bool after_own_ft, cudaStream_t stream) {
+  const int S = pl.KSL;
+  if (S <= 1) return run_fused_into(pl, x, u, y, after_own_ft, stream);
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) return cuda_fail("device");
+  ForkCtx* fc = fork_ctx(dev);
+  if (!fc) return I2CW_EINVAL;
+  std::lock_guard<std::mutex> lk(fc->mu);
+  if (!fc->ready) {
+    for (auto& st : fc->st)
+      if (cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking) != cudaSuccess) return cuda_fail("stream");
+    for (auto& e : fc->ev)
+      if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) return cuda_fail("event");
+    fc->ready = true;
+  }
+  const size_t ycount = (size_t)pl.N * pl.OD * pl.P * pl.Q * pl.K;
+  const size_t ystride = (ycount + 63) / 64 * 64;  // 256-byte aligned slices (TMA base alignment)
+  float* ws = nullptr;
+  if (cudaMallocAsync(&ws, (size_t)(S - 1) * ystride * 4, stream) != cudaSuccess) return cuda_fail("alloc");
+  const int per = cdiv(pl.NCC, S);
+  int rc = I2CW_OK;
+  if (cudaEventRecord(fc->ev[0], stream) != cudaSuccess) rc = cuda_fail("record");  // after U, workspace
+  for (int s = 0; s < S && rc == I2CW_OK; ++s) {
+    Plan ps = pl;
+    ps.CC0 = s * per;
+    ps.CC1 = std::min(pl.NCC, ps.CC0 + per);
+    ps.CPC = ps.CC1 - ps.CC0;
+    ps.NKC = 1;
+    ps.KSL = 1;
+    if (ps.CC0 >= ps.CC1) break;
+    cudaStream_t st = s == 0 ? stream : fc->st[s - 1];
+    if (s > 0 && cudaStreamWaitEvent(st, fc->ev[0], 0) != cudaSuccess) { rc = cuda_fail("fork"); break; }
+    rc = run_fused_into(ps, x, u, s == 0 ? y : ws + (size_t)(s - 1) * ystride, s == 0 && after_own_ft, st);
+    if (rc == I2CW_OK && s > 0 &&
+        (cudaEventRecord(fc->ev[s], st) != cudaSuccess || cudaStreamWaitEvent(stream, fc->ev[s], 0) != cudaSuccess))
+      rc = cuda_fail("join");
+  }
+  if (rc == I2CW_OK && launch_ksum(y, ws, S - 1, ycount, ystride, stream) != cudaSuccess) rc = cuda_fail("ksum");
+  cudaFreeAsync(ws, stream);
+  return rc;
 }
 
 int conv_plan(const Plan& plan, int is_deconv, const float* x, const float* w, float* y, cudaStream_t stream, bool simt,
@@ -928,6 +1020,7 @@ I2CW_API int i2cw_debug_conv_simt(int is_deconv, int N, int H, int W, int C, int
 // Longest TMEM accumulation in k-steps (0 restores the per-alpha default); returns the previous
 // setting (0 = default).
 I2CW_API int i2cw_debug_set_kchunk(int ksteps) { return g_kchunk_max.exchange(ksteps > 0 ? ksteps : 0); }
+I2CW_API int i2cw_debug_set_kslices(int n) { return g_kslices_max.exchange(n > 0 ? n : -1); }
 
 // Runs the product path with CTA 0's event timeline recorded into trace (device,
 // 32 kinds x 512 uint64 clock64 stamps; see trace_rec in common.cuh).
@@ -944,7 +1037,7 @@ I2CW_API int i2cw_debug_plan(int is_deconv, int N, int H, int W, int C, int K, i
   if (rc != I2CW_OK) return rc;
   int v[] = {pl.P, pl.Q, pl.m, pl.alpha, pl.NT, pl.NB, pl.NCC, pl.NKS, pl.T_r, pl.TS, pl.SEGS, pl.ROWS, pl.PB,
              pl.WBOX, pl.HBOX, pl.tile_blocks, pl.GP, pl.NPASS, pl.NUS, pl.smem_bytes, pl.pad_h, pl.pad_w, pl.NI,
-             pl.NFULL, pl.NITEMS, pl.pair, pl.NKC, pl.CPC};
+             pl.NFULL, pl.NITEMS, pl.pair, pl.NKC, pl.CPC, pl.KSL};
   for (int i = 0; i < 32; ++i) out[i] = i < (int)(sizeof(v) / sizeof(v[0])) ? v[i] : 0;
   return I2CW_OK;
 }

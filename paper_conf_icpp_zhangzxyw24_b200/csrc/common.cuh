@@ -44,6 +44,7 @@ struct Plan {
   int NKC, CPC;         // K-chunks (launches) of the K loop, channel chunks per K-chunk (bounded accumulation)
   int CC0, CC1;         // this launch's channel chunks [CC0, CC1) (set per K-chunk launch)
   int ACCUM;            // 1: every pass adds into y (a K-chunk after the first)
+  int KSL;              // concurrent K-slice launches (small grids, api.cu run_fused); 1: none
   int prec;             // 0: 3xTF32 (default, fp32 accuracy); 1: 1xTF32 (looser tolerance, f4)
   int NUS;              // U ring super-slots (KPS k-steps of GP points each)
   int OSB;              // bytes of one output staging buffer = NI*ROWS*TS*16*4 (TMA store box, 16 channels)

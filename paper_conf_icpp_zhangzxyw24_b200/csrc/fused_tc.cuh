@@ -190,6 +190,10 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
   // UW: each transform warpgroup checks its k-step's U super-slot (while it waits for its V slot
   // anyway) before arriving; the issuer's one wait per super-stage then covers V and U
   constexpr bool UW = I2CW_UWAIT_WG;
+#ifndef I2CW_ISS_LOOKAHEAD
+#define I2CW_ISS_LOOKAHEAD 0  // experiment: 1 = issuer waits for super-stage j+1 inside j's issue
+#endif
+  constexpr bool LA = I2CW_ISS_LOOKAHEAD && kps_for(A, NT) >= 2;
   constexpr uint32_t UBYTES = Cfg::UBYTES;
   const uint32_t rank = PAIR ? cluster_ctarank() : 0u;  // 0 = MMA leader
 
@@ -739,15 +743,23 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
           mbar_wait_tc<PAIR>(d_empty, (gpass - 1) & 1);
           tc_fence_after();
         }
+        // wait for super-stage (V and U) readiness; with LA the wait for the NEXT super-stage of
+        // the pass is done between this super-stage's two k-steps, while the tensor pipe still
+        // holds queued MMAs, so it no longer sits between two super-stages' issue phases
+        auto wait_ss = [&](int s_, int sp_, int u_, int up_) {
+          if constexpr (PAIR) {  // both CTAs' V (peer arrivals are remote) and both U halves
+            mbar_wait_cluster(&st_full[s_], sp_);
+            if constexpr (!UW) mbar_wait_cluster(&u_full[u_], up_);
+          } else {
+            mbar_wait(&st_full[s_], sp_);
+            if constexpr (!UW) mbar_wait(&u_full[u_], up_);
+          }
+        };
+        bool ready = false;  // this super-stage already waited for (LA lookahead)
         for (int kl0 = 0; kl0 < NKSP; kl0 += KPS, ++sgi) {
           trace_rec(pl.trace, 29, sgi, iss == 0 && lane32 == 0);
-          if constexpr (PAIR) {  // both CTAs' V (peer arrivals are remote) and both U halves
-            mbar_wait_cluster(&st_full[ss], sph);
-            if constexpr (!UW) mbar_wait_cluster(&u_full[us], uph);
-          } else {
-            mbar_wait(&st_full[ss], sph);
-            if constexpr (!UW) mbar_wait(&u_full[us], uph);
-          }
+          if (!ready) wait_ss(ss, sph, us, uph);
+          ready = false;
           tc_fence_after();
           trace_rec(pl.trace, 16, sgi, iss == 0 && lane32 == 0);
           if (!(ABL(2))) {  // DEBUG timing ablation: skip the MMAs (commits still signal)
@@ -780,6 +792,12 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
               }
               if constexpr (PAIR) mma_commit2_warp(sfree);
               else mma_commit_warp(sfree);
+              if (LA && pos == 0 && kl0 + KPS < NKSP) {  // lookahead: the next super-stage of this pass
+                const int s2 = ss + 1 == NSS ? 0 : ss + 1, sp2 = ss + 1 == NSS ? sph ^ 1 : sph;
+                const int u2 = us + 1 == NUS ? 0 : us + 1, up2 = us + 1 == NUS ? uph ^ 1 : uph;
+                wait_ss(s2, sp2, u2, up2);
+                ready = true;
+              }
             }
           } else {  // DEBUG ablation 2 (no MMAs): the slots are still released
 #pragma unroll

@@ -6,6 +6,8 @@
 * every residue Q mod m of every r = 2..9, conv and deconv;
 * K-chunked accumulation: the K loop split into chunks whose partial sums the
   TMA reduce-add combines, forced small with the i2cw_debug_set_kchunk test hook;
+* concurrent K slices on small grids (api.cu run_fused): parity, determinism, and the same
+  result as the unsliced path within the bound;
 * the mean relative error on U[1, 2] (the paper's Table 3 metric) held to the band measured
   on B200 (the tcgen05 fp32 accumulator truncates once per MMA), so a
   precision regression fails.
@@ -86,15 +88,46 @@ def test_k_chunks_reduce_truncation_error():
     """With all-positive inputs the truncating accumulator's error grows with the accumulation
     length; chunking the same K loop lowers the mean error."""
     args = ("conv", 2, 10, 24, 256, 64, 3, 3, 1, 1)
-    y1, yr, _ = run_case(*args, lo=1.0, hi=2.0)
-    old = i2cw.debug_set_kchunk(24)  # 96 k-steps -> 4 chunks of 24
+    oldsl = i2cw.debug_set_kslices(1)  # one accumulation (no concurrent K slices on this small grid)
     try:
-        y4, _, _ = run_case(*args, lo=1.0, hi=2.0)
+        y1, yr, _ = run_case(*args, lo=1.0, hi=2.0)
+        old = i2cw.debug_set_kchunk(24)  # 96 k-steps -> 4 chunks of 24
+        try:
+            y4, _, _ = run_case(*args, lo=1.0, hi=2.0)
+        finally:
+            i2cw.debug_set_kchunk(old)
     finally:
-        i2cw.debug_set_kchunk(old)
+        i2cw.debug_set_kslices(oldsl)
     e1, e4 = _mean_rel(y1, yr), _mean_rel(y4, yr)
     print(f"mean rel: one accumulation {e1:.3e}, 4 K-chunks {e4:.3e}")
     assert e4 < 0.6 * e1
+
+
+# 4 slices (alpha 12, 3 passes), 2 slices (CTA pairs, whole units; split tail), 3 slices (r = 7)
+KSLICE_CASES = [("conv", 1, 12, 20, 96, 64, 8, 4), ("conv", 1, 7, 7, 512, 512, 3, 1),
+                ("deconv", 1, 9, 11, 256, 64, 5, 2), ("conv", 1, 10, 10, 256, 128, 7, 3)]
+
+
+@pytest.mark.parametrize("kind,N,H,W,C,K,r,p", KSLICE_CASES, ids=lambda v: str(v))
+def test_k_slices_small_grid(kind, N, H, W, C, K, r, p):
+    """A per-GPU shard of a few images fills few SMs: the planner splits the K loop into
+    concurrent slices summed by a fixed-order combine. Every element within the
+    bound, bitwise repeatable, and close to the one-accumulation result."""
+    pl = i2cw.debug_plan(kind, N, H, W, C, K, r, r, p, p)
+    assert pl["KSL"] > 1, pl
+    y, yr, b = run_case(kind, N, H, W, C, K, r, r, p, p)
+    assert_parity(y, yr, b)
+    y2, _, _ = run_case(kind, N, H, W, C, K, r, r, p, p)
+    assert torch.equal(y, y2)
+    old = i2cw.debug_set_kslices(1)
+    try:
+        assert i2cw.debug_plan(kind, N, H, W, C, K, r, r, p, p)["KSL"] == 1
+        y1, _, _ = run_case(kind, N, H, W, C, K, r, r, p, p)
+    finally:
+        i2cw.debug_set_kslices(old)
+    assert_parity(y1, yr, b)
+    d = float((y.double().cpu() - y1.double().cpu()).abs().max())
+    assert d <= 2e-4 * float(b.max()), d
 
 
 # Mean relative error on U[1,2] (the paper's Table 3 metric) at C = K = 64 measured on B200 with
