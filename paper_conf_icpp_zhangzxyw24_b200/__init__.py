@@ -328,7 +328,7 @@ def transform_matrices(m, r, point_set=0):
 
 PLAN_FIELDS = ("P", "Q", "m", "alpha", "NT", "NB", "NCC", "NKS", "T_r", "TS", "SEGS", "ROWS", "PB", "WBOX", "HBOX",
                "tile_blocks", "GP", "NPASS", "NUS", "smem_bytes", "pad_h", "pad_w", "NI", "NFULL", "NITEMS", "pair",
-               "NKC", "CPC", "KSL")
+               "NKC", "CPC", "KSL", "NIS", "NOB", "PLANE")
 
 
 def debug_plan(kind, N, H, W, C, K, R, S, pad_h, pad_w):

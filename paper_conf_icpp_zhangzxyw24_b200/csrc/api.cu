@@ -1037,7 +1037,7 @@ I2CW_API int i2cw_debug_plan(int is_deconv, int N, int H, int W, int C, int K, i
   if (rc != I2CW_OK) return rc;
   int v[] = {pl.P, pl.Q, pl.m, pl.alpha, pl.NT, pl.NB, pl.NCC, pl.NKS, pl.T_r, pl.TS, pl.SEGS, pl.ROWS, pl.PB,
              pl.WBOX, pl.HBOX, pl.tile_blocks, pl.GP, pl.NPASS, pl.NUS, pl.smem_bytes, pl.pad_h, pl.pad_w, pl.NI,
-             pl.NFULL, pl.NITEMS, pl.pair, pl.NKC, pl.CPC, pl.KSL};
+             pl.NFULL, pl.NITEMS, pl.pair, pl.NKC, pl.CPC, pl.KSL, pl.NIS, pl.NOB, pl.PLANE};
   for (int i = 0; i < 32; ++i) out[i] = i < (int)(sizeof(v) / sizeof(v[0])) ? v[i] : 0;
   return I2CW_OK;
 }
