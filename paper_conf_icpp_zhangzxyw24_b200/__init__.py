@@ -328,12 +328,12 @@ def transform_matrices(m, r, point_set=0):
 
 PLAN_FIELDS = ("P", "Q", "m", "alpha", "NT", "NB", "NCC", "NKS", "T_r", "TS", "SEGS", "ROWS", "PB", "WBOX", "HBOX",
                "tile_blocks", "GP", "NPASS", "NUS", "smem_bytes", "pad_h", "pad_w", "NI", "NFULL", "NITEMS", "pair",
-               "NKC", "CPC", "KSL", "NIS", "NOB", "PLANE")
+               "NKC", "CPC", "KSL", "NIS", "NOB", "PLANE", "strip", "NSTRIP")
 
 
 def debug_plan(kind, N, H, W, C, K, R, S, pad_h, pad_w):
     """The host planner's launch plan (test hook, not in the public header)."""
-    out = (ctypes.c_int * 32)()
+    out = (ctypes.c_int * 40)()
     _check("i2cw_debug_plan", lib().i2cw_debug_plan(int(kind == "deconv"), N, H, W, C, K, R, S, pad_h, pad_w,
                                                     ctypes.addressof(out)))
     return dict(zip(PLAN_FIELDS, list(out)))

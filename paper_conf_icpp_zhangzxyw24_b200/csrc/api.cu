@@ -23,6 +23,9 @@ cudaError_t launch_filter_transform(const float* w, float* u, int C, int K, int 
                                     UTag* tag_dst, cudaStream_t stream);
 cudaError_t launch_fused_tc(const CUtensorMap& xmap, const CUtensorMap& ymap, const Plan& pl, const float* u,
                             cudaStream_t stream);
+struct alignas(64) YMaps { CUtensorMap m[4]; };  // fused_strip.cuh
+cudaError_t launch_fused_strip_a8(const CUtensorMap& xmap, const YMaps& ym, const Plan& pl, const float* u,
+                                  cudaStream_t stream);
 cudaError_t launch_zero_tail(float* y, size_t count, bool wait_first, cudaStream_t stream);
 cudaError_t launch_transpose(const float* in, float* out, int B, int rows, int cols, cudaStream_t stream);
 cudaError_t launch_ksum(float* y, const float* slices, int nslices, size_t count, size_t stride, cudaStream_t stream);
@@ -32,6 +35,7 @@ namespace {
 
 
 constexpr int kSmemBudget = 225 * 1024;
+constexpr int kStripLanes = 32;  // input rows per strip (one TMEM subpartition), fused_strip.cuh
 
 // Longest accumulation in one TMEM accumulator, in k-steps (8 channels x 1 filter row each).
 // The tcgen05 fp32 accumulator rounds toward zero once per MMA (3 MMAs per k-step in 3xTF32),
@@ -155,6 +159,86 @@ int num_sms() {
 
 }  // namespace
 
+// Strip kernel (fused_strip.cuh): one input-row transform per 8-channel chunk
+// serves all R filter rows through TMEM row shifts. A strip = one tile column of up to
+// 33 - R output rows (+ R - 1 halo input rows) in the 32 lanes of a TMEM subpartition; a unit =
+// 4 consecutive strips in (n, row block, tw) order. Used for the 2D 3xTF32 alpha = 8 single-CTA
+// plans (the U layout of the pair plans differs) when its lane use is not much worse than the
+// base block shape's. I2CW_STRIP=0/1 disables / forces it (experiments).
+void plan_strip(Plan* plp, int nsm) {
+  Plan& pl = *plp;
+  static const int env = [] { const char* e = getenv("I2CW_STRIP"); return e ? atoi(e) : -1; }();
+  pl.strip = 0;
+  if (env == 0 || pl.vol || pl.prec || pl.pair || pl.alpha != 8 || pl.NT != 64 || pl.R > 24) return;
+  const int rbmax = 33 - pl.R;
+  const int pb = cdiv(pl.P, rbmax), rb = cdiv(pl.P, pb);
+  const long long nstrip = (long long)pl.N * pb * pl.T_r;
+  if (nstrip > (1 << 30)) return;
+  const int sgroups = (int)cdiv((int)nstrip, 4);
+  // lanes doing useful output work: strip plan vs the base plan's tile blocks
+  const double useful = (double)pl.N * pl.P * pl.T_r;
+  const double util_strip = useful / ((double)sgroups * kMaxLanes);
+  const double util_base = useful / ((double)pl.tile_blocks * kMaxLanes);
+  if (env != 1 && util_strip < 0.85 * util_base) return;
+  constexpr int kUB = 4 * 2 * 64 * 32, kStage = 4 * 9 * 32 * 32;  // U k-step, 4 strip boxes (alpha = 8)
+  const int osb = 4 * 2048, ostride = osb;  // 4 strips x 32 rows x 16 channels per output buffer
+  // (U k-step slots, input stages, output buffers >= 2)
+  static int kSD[][3] = {{8, 2, 2}, {6, 2, 2}, {5, 2, 2}, {4, 2, 2}, {3, 2, 2}, {2, 2, 2}};
+  static const bool sd_env = [] {  // I2CW_STRIP_DEPTHS=u,i,o (experiments): try these first
+    const char* e = getenv("I2CW_STRIP_DEPTHS");
+    int a, b, c;
+    if (e && sscanf(e, "%d,%d,%d", &a, &b, &c) == 3 && b >= 1 && c >= 2) { kSD[0][0] = a; kSD[0][1] = b; kSD[0][2] = c; }
+    return e != nullptr;
+  }();
+  (void)sd_env;
+  int sel = -1, smem = 0;
+  for (int d = 0; d < (int)(sizeof(kSD) / sizeof(kSD[0])); ++d) {
+    const int bar_bytes = 8 * (4 + kSD[d][1] + 10 + 2 * kSD[d][0]) + 16;
+    smem = kSD[d][0] * kUB + kSD[d][1] * kStage + 4 * kSD[d][2] * ostride + bar_bytes;
+    if (smem <= kSmemBudget) { sel = d; break; }
+  }
+  if (sel < 0) return;
+  pl.strip = 1;
+  pl.NSTRIP = (int)nstrip;
+  pl.ROWS = rb;
+  pl.PB = pb;
+  pl.TS = 4;
+  pl.NI = 1;
+  pl.SEGS = 1;
+  pl.HBOX = kStripLanes;
+  pl.WBOX = pl.alpha;
+  pl.tile_blocks = sgroups;
+  pl.NUS = kSD[sel][0];
+  pl.NIS = kSD[sel][1];
+  pl.NOB = kSD[sel][2];
+  pl.OSB = osb;
+  pl.OSTRIDE = ostride;
+  pl.BOXB = kStage;
+  pl.PLANE = kStage / 2;
+  pl.smem_bytes = smem;
+  std::fill(pl.lane_row, pl.lane_row + kMaxLanes, 0);
+  std::fill(pl.lane_in, pl.lane_in + kMaxLanes, 0);
+  std::fill(pl.lane_tw, pl.lane_tw + kMaxLanes, 0);
+  const int units = sgroups * pl.NB;
+  const int tail = units % nsm;
+  const char* st = getenv("I2CW_SPLIT_TAIL");
+  static const bool allsplit = [] { const char* e = getenv("I2CW_STRIP_ALLSPLIT"); return e && e[0] == '1'; }();
+  if (pl.NPASS == 2 && allsplit) {  // experiments: every unit as two one-pass items
+    pl.NFULL = 0;
+    pl.NITEMS = 2 * units;
+  } else if (pl.NPASS == 2 && !(st && st[0] == '0') && tail > 0 && 2 * tail <= nsm) {
+    pl.NFULL = units - tail;
+    pl.NITEMS = pl.NFULL + 2 * tail;
+  } else {
+    pl.NFULL = pl.NITEMS = units;
+  }
+  const int item_ksteps = pl.NKS * (pl.NFULL > 0 ? pl.NPASS : 1);
+  pl.KSL = 1;
+  if (pl.NKC == 1 && pl.NCC >= 2 && 2 * pl.NITEMS <= nsm)
+    pl.KSL = std::max(1, std::min({kslices_cap(), pl.NCC, nsm / std::max(1, pl.NITEMS), item_ksteps / 64}));
+  if (pl.KSL > 1) pl.KSL = cdiv(pl.NCC, cdiv(pl.NCC, pl.KSL));
+}
+
 // Build the launch plan. Returns I2CW_OK or an error code.
 // vol = 1: 3D convolution (D, T, pad_d); 2D calls pass D = T = 1, pad_d = 0, vol = 0.
 int make_plan_uncached(int N, int D, int H, int W, int C, int K, int T, int R, int S, int pad_d, int pad_h, int pad_w,
@@ -165,7 +249,8 @@ int make_plan_uncached(int N, int D, int H, int W, int C, int K, int T, int R, i
       pad_h < 0 || pad_w < 0)
     return I2CW_EINVAL;
   if (!vol && (D != 1 || T != 1 || pad_d != 0)) return I2CW_EINVAL;
-  if (prec != 0 && prec != 1) return I2CW_EINVAL;
+  const int nostrip = prec & 2;
+  prec &= 1;
   if (prec && vol) return I2CW_EUNSUPPORTED;  // 1xTF32 kernels: 2D only
   Choice ch;
   if (!choose(S, C, &ch)) return I2CW_EUNSUPPORTED;
@@ -356,6 +441,7 @@ int make_plan_uncached(int N, int D, int H, int W, int C, int K, int T, int R, i
       pl.KSL = std::max(1, std::min({kslices_cap(), pl.NCC, nsm / std::max(1, ctas), item_ksteps / 64}));
     if (pl.KSL > 1) pl.KSL = cdiv(pl.NCC, cdiv(pl.NCC, pl.KSL));  // no empty slice
   }
+  if (!nostrip) plan_strip(&pl, nsm);  // prec bit 1: base plan only (the SIMT stepping stone)
   *out = pl;
   return I2CW_OK;
 }
@@ -429,6 +515,40 @@ int encode_x_map(const Plan& pl, const float* x, CUtensorMap* map) {
   cuuint32_t es[4] = {1, 1, 1, 1};
   CUresult r = enc(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, const_cast<float*>(x), dims, strides, box, es,
                    CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_32B, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS ? I2CW_OK : I2CW_EUNSUPPORTED;
+}
+
+// strip kernel: x box = 8 channels x (alpha + 1) columns x 32 rows, 32B swizzle: the 288-byte
+// row stride puts the 8 rows a quarter-warp reads in 8 distinct 16-byte bank groups
+// (tools/tma_view_test.cu checks the layout; a (C, H, W, N) view with non-monotonic strides
+// encodes but faults in the TMA unit)
+int encode_x_map_strip(const Plan& pl, const float* x, CUtensorMap* map) {
+  PFN_encodeTiled_t enc = get_encode();
+  if (!enc) return I2CW_ECUDA;
+  cuuint64_t dims[4] = {(cuuint64_t)pl.C, (cuuint64_t)pl.W, (cuuint64_t)pl.H, (cuuint64_t)pl.N};
+  cuuint64_t strides[3] = {(cuuint64_t)pl.C * 4, (cuuint64_t)pl.W * pl.C * 4, (cuuint64_t)pl.H * pl.W * pl.C * 4};
+  cuuint32_t box[4] = {8, (cuuint32_t)(pl.alpha + 1), (cuuint32_t)kStripLanes, 1};
+  cuuint32_t es[4] = {1, 1, 1, 1};
+  CUresult r = enc(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, const_cast<float*>(x), dims, strides, box, es,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_32B, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS ? I2CW_OK : I2CW_EUNSUPPORTED;
+}
+
+// strip kernel: y store box for a run of L strips = 16 channels x L tiles (element stride m) x ROWS
+// rows x 1 image; swizzle 64B for L = 3, else 128B (the staging writes of a warp -- 8 rows of one
+// tile -- are then conflict-free or 2-way, fused_strip.cuh). A box that starts at a negative
+// column faults (tools/tma_view_test.cu), hence one map per run length.
+int encode_y_map_strip(const Plan& pl, float* y, int L, CUtensorMap* map) {
+  PFN_encodeTiled_t enc = get_encode();
+  if (!enc) return I2CW_ECUDA;
+  cuuint64_t dims[4] = {(cuuint64_t)pl.K, (cuuint64_t)pl.Q, (cuuint64_t)pl.P, (cuuint64_t)pl.N};
+  cuuint64_t strides[3] = {(cuuint64_t)pl.K * 4, (cuuint64_t)pl.Q * pl.K * 4, (cuuint64_t)pl.P * pl.Q * pl.K * 4};
+  cuuint32_t box[4] = {16, (cuuint32_t)(L * pl.m), (cuuint32_t)pl.ROWS, 1};
+  cuuint32_t es[4] = {1, (cuuint32_t)pl.m, 1, 1};
+  CUresult r = enc(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, y, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                   CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_NONE,
                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   return r == CUDA_SUCCESS ? I2CW_OK : I2CW_EUNSUPPORTED;
 }
@@ -582,15 +702,22 @@ int run_fused_into(const Plan& pl, const float* x, const void* u, float* y, bool
     // image the tail touches (earlier rows of that image are overwritten by whole-unit stores)
     const int tb0 = (pl.pair ? 2 : 1) * (pl.NFULL / pl.NB);  // first tile block of the tail
     const int ib = tb0 / pl.SEGS / pl.PB;  // image block of the first tail unit
-    const size_t n0 = pl.vol ? (size_t)(ib / pl.DB) : (size_t)ib * pl.NI;
+    size_t n0 = pl.vol ? (size_t)(ib / pl.DB) : (size_t)ib * pl.NI;
+    if (pl.strip) n0 = (size_t)((long long)tb0 * 4 / pl.T_r / pl.PB);  // image of the tail's first strip
     const size_t img = (size_t)pl.OD * pl.P * pl.Q * pl.K;
     if (n0 < (size_t)pl.N &&
         launch_zero_tail(y + n0 * img, ((size_t)pl.N - n0) * img, !after_own_ft, stream) != cudaSuccess)
       return cuda_fail("zero tail");
   }
-  int rc = encode_x_map(pl, x, &map);
+  YMaps ym;
+  int rc = pl.strip ? encode_x_map_strip(pl, x, &map) : encode_x_map(pl, x, &map);
   if (rc != I2CW_OK) return rc;
-  if ((rc = encode_y_map(pl, y, &ymap)) != I2CW_OK) return rc;
+  if (pl.strip) {
+    for (int L = 1; L <= 4; ++L)
+      if ((rc = encode_y_map_strip(pl, y, L, &ym.m[L - 1])) != I2CW_OK) return rc;
+  } else if ((rc = encode_y_map(pl, y, &ymap)) != I2CW_OK) {
+    return rc;
+  }
   const float* ud = reinterpret_cast<const float*>(static_cast<const uint8_t*>(u) + kUTagBytes);
   // K-chunks: one launch per chunk of <= CPC channel chunks, in order on the
   // stream; the first stores y (its split tail reduce-adds into the zeroed region), later ones
@@ -603,7 +730,9 @@ int run_fused_into(const Plan& pl, const float* x, const void* u, float* y, bool
     // the split tail's two one-pass items per unit add in either order: exact only onto y = 0
     // (0 + a + b), so later chunks (y != 0) run every unit whole, its passes in order
     if (kc > 0) pk.NFULL = pk.NITEMS = pl.NFULL + (pl.NITEMS - pl.NFULL) / 2;
-    if (launch_fused_tc(map, ymap, pk, ud, stream) != cudaSuccess) return cuda_fail("fused launch");
+    const cudaError_t e = pl.strip ? (pl.alpha == 8 ? launch_fused_strip_a8(map, ym, pk, ud, stream) : cudaErrorInvalidValue)
+                                   : launch_fused_tc(map, ymap, pk, ud, stream);
+    if (e != cudaSuccess) return cuda_fail("fused launch");
   }
   return I2CW_OK;
 }
@@ -678,7 +807,9 @@ int conv_common(int is_deconv, int N, int H, int W, int C, int K, int R, int S, 
   if (!x || !w || !y) return I2CW_EINVAL;
   if (!aligned16(x) || !aligned16(w) || !aligned16(y)) return I2CW_EINVAL;
   Plan pl;
-  int rc = make_plan(N, H, W, C, K, R, S, pad_h, pad_w, is_deconv, &pl);
+  // the SIMT stepping stone reads the base plan's block shape
+  int rc = simt ? make_plan3(N, 1, H, W, C, K, 1, R, S, 0, pad_h, pad_w, is_deconv, 0, &pl, 2)
+                : make_plan(N, H, W, C, K, R, S, pad_h, pad_w, is_deconv, &pl);
   if (rc != I2CW_OK) return rc;
   return conv_plan(pl, is_deconv, x, w, y, stream, simt, trace);
 }
@@ -1031,14 +1162,14 @@ I2CW_API int i2cw_debug_trace(int is_deconv, int N, int H, int W, int C, int K, 
 }
 
 I2CW_API int i2cw_debug_plan(int is_deconv, int N, int H, int W, int C, int K, int R, int S, int pad_h, int pad_w,
-                    int* out /* 32 ints */) {
+                    int* out /* 40 ints */) {
   Plan pl;
   int rc = make_plan(N, H, W, C, K, R, S, pad_h, pad_w, is_deconv, &pl);
   if (rc != I2CW_OK) return rc;
   int v[] = {pl.P, pl.Q, pl.m, pl.alpha, pl.NT, pl.NB, pl.NCC, pl.NKS, pl.T_r, pl.TS, pl.SEGS, pl.ROWS, pl.PB,
              pl.WBOX, pl.HBOX, pl.tile_blocks, pl.GP, pl.NPASS, pl.NUS, pl.smem_bytes, pl.pad_h, pl.pad_w, pl.NI,
-             pl.NFULL, pl.NITEMS, pl.pair, pl.NKC, pl.CPC, pl.KSL, pl.NIS, pl.NOB, pl.PLANE};
-  for (int i = 0; i < 32; ++i) out[i] = i < (int)(sizeof(v) / sizeof(v[0])) ? v[i] : 0;
+             pl.NFULL, pl.NITEMS, pl.pair, pl.NKC, pl.CPC, pl.KSL, pl.NIS, pl.NOB, pl.PLANE, pl.strip, pl.NSTRIP};
+  for (int i = 0; i < 40; ++i) out[i] = i < (int)(sizeof(v) / sizeof(v[0])) ? v[i] : 0;
   return I2CW_OK;
 }
 

@@ -5,6 +5,7 @@
 #include <cuda.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <cstdio>
 
 #ifndef I2CW_ABLATION
 #define I2CW_ABLATION 0  // 1: timing-ablation branches compiled in (make ABLATION=1; tools only)
@@ -53,6 +54,9 @@ struct Plan {
   int NIS;              // input (x row box) stages
   int smem_bytes;
   int pair;             // 1: CTA pairs (cluster of 2) with tcgen05.mma.cta_group::2, U split by N halves
+  int strip;            // 1: strip kernel (fused_strip.cuh): one input-row transform per chunk, TMEM row
+                        // shifts between filter rows; ROWS = valid rows per strip, TS = 4 strips per unit
+  int NSTRIP;           // strip kernel: strips = N * PB * T_r (tile column tw fastest)
   int ablate;           // DEBUG timing ablation (I2CW_ABLATE, results wrong): 1 no transform math,
                         // 2 no MMAs, 4 no epilogue math/stores; 0 in production
   unsigned long long* trace;  // debug timeline of CTA 0 (nullptr = off), see i2cw_debug_trace
@@ -200,11 +204,19 @@ __device__ __forceinline__ bool mbar_try_wait(uint64_t* bar, uint32_t parity) {
 }
 // Blocking wait with a watchdog: a protocol bug traps (launch error) after ~4 s
 // instead of hanging the GPU.
+#ifndef I2CW_WATCHDOG_PRINT
+#define I2CW_WATCHDOG_PRINT 0  // debug builds: report the stuck barrier before trapping
+#endif
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
   if (mbar_try_wait(bar, parity)) return;
   const uint64_t t0 = globaltimer();
   while (!mbar_try_wait(bar, parity)) {
-    if (globaltimer() - t0 > 4000000000ull) __trap();
+    if (globaltimer() - t0 > 4000000000ull) {
+#if I2CW_WATCHDOG_PRINT
+      printf("i2cw watchdog: block %d thread %d smem bar 0x%x parity %u\n", blockIdx.x, threadIdx.x, smem_u32(bar), parity);
+#endif
+      __trap();
+    }
   }
 }
 

@@ -1,0 +1,521 @@
+// Strip variant of the fused Im2col-Winograd kernel (rows a2-a5 of SURVEY.md §8(a)):
+// one input-row transform per channel chunk serves all R filter rows, through tcgen05.shift.
+//
+// Method (§4.1, Fig 2): for tile (n, p, q0) and filter row fh,
+//   V_t[(fh,c)] = sum_j BT[t][j] x[n][p-ph+fh][q0-pw+j][c]
+// depends on (p, fh) only through the input row rho = p + fh: V_t[(fh,c)](p) = V'_t[c](p + fh).
+// The base kernel (fused_tc.cuh) computes V once per (tile, fh), i.e. each input row's
+// transform R times. Here a "strip" is one tile column tw of SL <= 32 consecutive input rows
+// held by the 32 TMEM lanes of one subpartition (lane j <-> input row rb*RB - ph + j); each lane
+// transforms its own row ONCE per 8-channel chunk. The MMAs of filter row fh need lane j to hold
+// row j + fh: between filter rows the issuer shifts the V slot up by one lane
+// (tcgen05.shift.cta_group::1.down: lane l <- lane l+1 inside each 32-lane subpartition,
+// executed in order with the MMAs; tools/shift_bench.cu measured its semantics, ordering and
+// ~8-12 cycles per 32-byte column block inside an MMA stream). Lanes j < RB = SL - (R-1) are
+// output rows; lanes j >= RB only feed their input rows to the shift (their outputs are never
+// stored). Accumulation over fh and c, the output transform y = A^T M and the boundary
+// (TMA clipping) are the base kernel's.
+//
+// Work unit = (strip group sg, output-channel block nb): the 4 consecutive strips 4sg..4sg+3 in
+// (n, rb, tw) order, one per subpartition. k-step ks = (channel chunk cc, filter row fh) as in
+// the base kernel (same U layout); the V ring holds one CHUNK per slot (R k-steps of MMAs per V).
+// Warp roles as the base kernel: 4 transform/epilogue warpgroups (WG g owns the chunks gc = g mod
+// 4 and V slot g), one input-TMA warp, one U-ring warp, two MMA issuer warps.
+#pragma once
+#include "fused_tc.cuh"
+
+namespace i2cw {
+
+__device__ __forceinline__ void tmem_shift_up_warp(uint32_t taddr) {
+  // PTX ".down" moves each row's 32-byte element to the row below in the matrix view, i.e. lane l
+  // receives lane l+1's value (measured, tools/shift_bench.cu); one elected lane issues
+  asm volatile(
+      "{\n\t.reg .pred e;\n\t"
+      "elect.sync _|e, 0xffffffff;\n\t"
+      "@e tcgen05.shift.cta_group::1.down [%0];\n\t}" ::"r"(taddr)
+      : "memory");
+}
+
+constexpr int kStripLanes = 32;  // input rows per strip box (one TMEM subpartition)
+struct alignas(64) YMaps { CUtensorMap m[4]; };  // y store maps for runs of 1..4 strips
+
+template <int M, int RW>
+struct StripCfg {
+  using T = Wino<M, RW>;
+  static constexpr int A = T::alpha;
+  static constexpr int NT = 64;
+  static constexpr int GP = gp_for(A, NT);  // points per pass
+  static constexpr int NPASS = A / GP;
+  static constexpr int NWG = 4;
+  static constexpr int NSLOT = 4;           // V slots (one chunk each, one per warpgroup)
+  static constexpr int NISS = niss_for(GP);
+  static constexpr int PPI = GP / NISS;
+  static constexpr int VCOL = GP * NT;
+  static constexpr int UBYTES = GP * 2 * NT * 32;                // one k-step of U (GP points, hi + lo)
+  // one strip's input box: 8 ch x (A + 1) cols x 32 rows, smem image [row][col][8 ch] with the TMA
+  // 32B swizzle; the 9th column makes the row stride 288 B, so 8 consecutive rows read 8 distinct
+  // 16-byte bank groups (a 256-byte stride with any swizzle leaves 2-way conflicts)
+  static constexpr int WCOL = A + 1;
+  static constexpr int SBOX = WCOL * kStripLanes * 32;
+  static constexpr int NTHREADS = NWG * 128 + 64 + NISS * 32;
+  static_assert(GP * NT + NSLOT * GP * 16 <= 512, "TMEM budget");
+  static_assert(SBOX % 1024 == 0, "boxes stay 1024-aligned");
+  static constexpr int TSTRIDE = 2048;  // y staging bytes per strip (32 rows x 64 B)
+};
+
+// Plan fields used: strip layout NSTRIP, ROWS (= RB valid rows per strip), PB, T_r, NB; rings
+// NUS (U k-step slots), NIS (input stages of 4 strip boxes), NOB, OSTRIDE; items NFULL/NITEMS;
+// K-chunk CC0/CC1/ACCUM. xmap: x (C, W, H, N) with box (8, A + 1, 32, 1), 32B swizzle
+// (tools/tma_view_test.cu checks the layout). ym.m[L-1]: y (K, Q, P, N) with box (16 ch, L tiles
+// at element stride m, ROWS rows, 1 image): one TMA op per run of L strips with the same (n, rb)
+// per output column (a box may not start at a negative column, so a run that starts inside the
+// unit needs its exact length); swizzle 64B for L = 3, else 128B (conflict-free or 2-way
+// staging writes).
+template <int M, int RW>
+__global__ void __launch_bounds__(StripCfg<M, RW>::NTHREADS, 1)
+    fused_strip_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__ YMaps ym,
+                       const __grid_constant__ Plan pl, const float* __restrict__ u) {
+  using Cfg = StripCfg<M, RW>;
+  using T = typename Cfg::T;
+  constexpr int A = Cfg::A, GP = Cfg::GP, NPASS = Cfg::NPASS, NWG = Cfg::NWG, NSLOT = Cfg::NSLOT;
+  constexpr int NISS = Cfg::NISS, PPI = Cfg::PPI, VCOL = Cfg::VCOL, NT = Cfg::NT;
+  constexpr uint32_t UBYTES = Cfg::UBYTES, SBOX = Cfg::SBOX;
+  constexpr int CPW = NT / NWG;  // epilogue channels per warpgroup (64-byte staging rows)
+  const int NIS = pl.NIS, NUS = pl.NUS, R = pl.R;
+
+  extern __shared__ __align__(1024) uint8_t smem[];
+  uint8_t* u_smem = smem;                                        // [NUS][UBYTES]
+  uint8_t* o_smem = u_smem + (size_t)NUS * UBYTES;               // [NWG][NOB][OSTRIDE]
+  uint8_t* in_smem = o_smem + (size_t)NWG * pl.NOB * pl.OSTRIDE;  // [NIS][4][SBOX]
+  uint64_t* bars = reinterpret_cast<uint64_t*>(in_smem + (size_t)NIS * 4 * SBOX);
+  // Input ring: the data stages rotate with gc mod NIS, but "chunk gc landed" is signalled on
+  // in_full[gc mod 4], the consuming warpgroup's own barrier. A warpgroup consumes every 4th chunk
+  // and its 4 warps are not synchronised with each other, so a per-stage full barrier could be
+  // waited on two phases ahead (parity waits alias phase k and k - 2: measured as stale boxes).
+  // Per warpgroup, each warp waits every phase of its barrier in order.
+  uint64_t* in_full = bars;              // [4]
+  uint64_t* in_empty = in_full + 4;      // [NIS]
+  uint64_t* st_full = in_empty + NIS;    // [NSLOT]
+  uint64_t* st_empty = st_full + NSLOT;  // [NSLOT]
+  uint64_t* d_full = st_empty + NSLOT;   // [1]
+  uint64_t* d_empty = d_full + 1;        // [1]
+  uint64_t* u_full = d_empty + 1;        // [NUS]
+  uint64_t* u_empty = u_full + NUS;      // [NUS]
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(u_empty + NUS);
+
+  const int warp = threadIdx.x / 32, lane32 = threadIdx.x % 32;
+  const int NITEMS = pl.NITEMS;
+  struct Item { int ui, pb, pe; bool split; };
+  auto item_at = [&](int it) {
+    Item I;
+    if (it < pl.NFULL) { I.ui = it; I.pb = 0; I.pe = NPASS; I.split = false; }
+    else { const int h = it - pl.NFULL; I.ui = pl.NFULL + h / 2; I.pb = h % 2; I.pe = I.pb + 1; I.split = true; }
+    return I;
+  };
+  struct Strip { int n, rb, tw; };
+  auto strip_at = [&](int sg) {  // strip index -> (image, row block, tile column); tw fastest
+    Strip s;
+    s.tw = sg % pl.T_r;
+    const int r = sg / pl.T_r;
+    s.rb = r % pl.PB;
+    s.n = r / pl.PB;
+    return s;
+  };
+  const int CC0 = pl.CC0, NCCL = pl.CC1 - pl.CC0;
+  auto crot_of = [&](int ui) { return (int)(((unsigned)ui * 5u) % (unsigned)NCCL); };
+  auto chunk_of = [&](int ui, int cc) {  // actual channel chunk of the unit's cc-th chunk (rotated)
+    const int cr = crot_of(ui);
+    return CC0 + (cc + cr < NCCL ? cc + cr : cc + cr - NCCL);
+  };
+  constexpr int PROD_WARP = NWG * 4, UPROD_WARP = PROD_WARP + 1, ISS_WARP0 = NWG * 4 + 2;
+
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < 4; ++i) mbar_init(&in_full[i], 1);
+    for (int i = 0; i < NIS; ++i) mbar_init(&in_empty[i], 4);
+    for (int i = 0; i < NSLOT; ++i) { mbar_init(&st_full[i], 4); mbar_init(&st_empty[i], NISS); }
+    for (int i = 0; i < NUS; ++i) { mbar_init(&u_full[i], 1); mbar_init(&u_empty[i], NISS); }
+    mbar_init(d_full, NISS);
+    mbar_init(d_empty, NWG * 4);
+    fence_mbar_init();
+  }
+  if (warp == ISS_WARP0) { tmem_alloc(tmem_slot, 512); tmem_relinquish(); }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tbase = *tmem_slot;
+
+  if (warp < NWG * 4) {
+    setmaxnreg_inc<104>();
+    // ===================== transform + epilogue warpgroups =====================
+    const int g = warp / 4;           // chunks gc = g (mod 4), V slot g
+    const int sub = warp % 4;         // TMEM subpartition = strip of the unit
+    const int l = threadIdx.x % 128;  // TMEM lane
+    const int jr = lane32;            // input row of the strip box held by this lane
+    const uint32_t lane_addr = tbase + ((uint32_t)(l & ~31) << 16);
+    const uint32_t vslot = lane_addr + VCOL + (uint32_t)g * GP * 16;
+    const uint32_t rofs = (uint32_t)jr * (Cfg::WCOL * 32);  // this lane's row in the box
+    const bool out_row = jr < pl.ROWS;  // output row of the strip (else: halo input row only)
+    uint8_t* ostage = o_smem + (size_t)g * pl.NOB * pl.OSTRIDE;
+    // ---- one chunk of V (this warpgroup's chunk gc of a pass with point group PASS) ----
+    auto do_chunk = [&](auto PASS_, int gc) {
+      constexpr int PASS = PASS_;
+      const int ist = gc % NIS;
+      trace_rec(pl.trace, 0 + g, gc / NWG, l == 0);
+      mbar_wait(&in_full[g], (gc / NWG) & 1);
+      trace_rec(pl.trace, 4 + g, gc / NWG, l == 0);
+      const uint8_t* box = in_smem + ((size_t)ist * 4 + sub) * SBOX;
+      float2 V[GP][4];  // point tl, channel pair cp
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        float2 d[A][2];
+#pragma unroll
+        for (int j = 0; j < A; ++j) {
+          const uint32_t o = rofs + (uint32_t)j * 32;  // 32B swizzle: bit 4 ^= bit 7
+          const float4 v = *reinterpret_cast<const float4*>(box + ((o ^ ((o >> 3) & 16u)) ^ (uint32_t)(h << 4)));
+          d[j][0] = make_float2(v.x, v.y);
+          d[j][1] = make_float2(v.z, v.w);
+        }
+        static_for<GP / 2>([&](auto Q_) {
+          constexpr int idx0 = PASS * GP + 2 * (int)Q_;
+          constexpr int tl0 = 2 * (int)Q_;
+#pragma unroll
+          for (int p = 0; p < 2; ++p) {
+            if constexpr (idx0 == 0) {
+              V[tl0][2 * h + p] = bt_dot2<T, 0, 1, 0>(d, p);
+              V[tl0 + 1][2 * h + p] = bt_dot2<T, A - 1, 1, 0>(d, p);
+            } else {
+              constexpr int pa = point_of(idx0, A);
+              const float2 E = bt_dot2<T, pa, 2, 0>(d, p);
+              const float2 O = bt_dot2<T, pa, 2, 1>(d, p);
+              V[tl0][2 * h + p] = __fadd2_rn(E, O);
+              V[tl0 + 1][2 * h + p] = __ffma2_rn(make_float2(-1.f, -1.f), O, E);
+            }
+          }
+        });
+      }
+      // Release the box once every load of this lane has completed: the branch reads a sum of
+      // all 16 loaded vectors (an arrive issued right after the LDS instructions can overtake
+      // them -- ptxas adds no wait -- and the next TMA fill would land under the reads). The
+      // bit pattern is a signalling NaN, which no sum produces, so the branch is always taken.
+      {
+        float2 acc2 = make_float2(0.f, 0.f);
+#pragma unroll
+        for (int t = 0; t < GP; ++t)
+#pragma unroll
+          for (int cp = 0; cp < 4; ++cp) acc2 = __fadd2_rn(acc2, V[t][cp]);
+        if (__float_as_uint(acc2.x + acc2.y) != 0x7f800001u) {
+          __syncwarp();
+          if (lane32 == 0) mbar_arrive(&in_empty[ist]);
+        }
+      }
+      trace_rec(pl.trace, 8 + g, gc / NWG, l == 0);
+      const int use = gc / NSLOT;
+      if (use > 0) mbar_wait(&st_empty[g], (use - 1) & 1);
+      trace_rec(pl.trace, 12 + g, gc / NWG, l == 0);
+      tc_fence_after();
+#pragma unroll
+      for (int t = 0; t < GP; ++t) {
+        float v16[16];
+#pragma unroll
+        for (int cp = 0; cp < 4; ++cp) {
+          float2 hi, lo;
+          split_tf32x2(V[t][cp], hi, lo);
+          v16[2 * cp] = hi.x; v16[2 * cp + 1] = hi.y;
+          v16[8 + 2 * cp] = lo.x; v16[8 + 2 * cp + 1] = lo.y;
+        }
+        tmem_st_x16(vslot + t * 16, v16);
+      }
+      tmem_wait_st();
+      tc_fence_before();
+      __syncwarp();
+      if (lane32 == 0) mbar_arrive(&st_full[g]);
+      trace_rec(pl.trace, 16 + g, gc / NWG, l == 0);
+    };
+
+    // ---- epilogue of one pass: y (+)= A^T M via shared memory + TMA ----
+    struct Epi { int gpass, pass, sg0, nb; bool split; };
+    auto do_epilogue = [&](auto PASS_, const Epi& E) {
+      constexpr int PASS = PASS_;
+      // runs of the unit: strips with the same (n, rb) (a run starts at s = 0 or where tw = 0).
+      // This warp's strip sub is tile t = sub - r0 of the run [r0, r0 + rl); the run's staging
+      // region starts at r0 * TSTRIDE and holds [row][rl tiles][16 ch] (the box image of map rl)
+      const int nvalid = min(4, pl.NSTRIP - E.sg0);
+      int r0 = 0, rl = 1;
+      for (int s = 1; s <= sub; ++s)
+        if (s < nvalid && strip_at(E.sg0 + s).tw == 0) r0 = s;
+      while (r0 + rl < nvalid && strip_at(E.sg0 + r0 + rl).tw != 0) ++rl;
+      // staging offset of this lane's row (bytes, before the swizzle) and the swizzle of map rl
+      // (64B for rl = 3: chunk bits [5:4] ^= [8:7]; else 128B: [6:4] ^= [9:7])
+      const uint32_t obase = (uint32_t)(r0 * Cfg::TSTRIDE + (jr * rl + (sub - r0)) * 64);
+      const uint32_t oxor = ((obase >> 7) & 3u) << 4;
+      const bool live = out_row && sub < nvalid;
+      trace_rec(pl.trace, 20 + g, 2 * E.gpass, l == 0);
+      mbar_wait(d_full, E.gpass & 1);
+      trace_rec(pl.trace, 20 + g, 2 * E.gpass + 1, l == 0);
+      tc_fence_after();
+      const int cbase = g * CPW;
+      float mv[GP][CPW];
+#pragma unroll
+      for (int t = 0; t < GP; ++t) tmem_ld_x16(lane_addr + t * NT + cbase, &mv[t][0]);
+      tmem_wait_ld();
+      tc_fence_before();
+      __syncwarp();
+      if (lane32 == 0) mbar_arrive(d_empty);  // accumulators read: the next pass's MMAs may start
+      static_for<GP / 2>([&](auto Q_) {  // pair (a, a+1): AT[i][a+1] = (-1)^i AT[i][a]
+        constexpr int idx0 = PASS * GP + 2 * (int)Q_;
+        constexpr int tl0 = 2 * (int)Q_;
+        if constexpr (idx0 != 0) {
+#pragma unroll
+          for (int e = 0; e < CPW; e += 2) {
+            const float2 a = make_float2(mv[tl0][e], mv[tl0][e + 1]), b = make_float2(mv[tl0 + 1][e], mv[tl0 + 1][e + 1]);
+            const float2 sa = __fadd2_rn(a, b), da = __ffma2_rn(make_float2(-1.f, -1.f), b, a);
+            mv[tl0][e] = sa.x; mv[tl0][e + 1] = sa.y;
+            mv[tl0 + 1][e] = da.x; mv[tl0 + 1][e + 1] = da.y;
+          }
+        }
+      });
+      trace_rec(pl.trace, 28 + (g == 0 ? 3 : 0), 0, false);
+      if (l == 0) {
+        bulk_wait_group_read_dyn(pl.NOB - 1);
+        if (PASS > 0 && !E.split) bulk_wait_group_all();  // the pass-0 stores of this unit landed
+      }
+      named_bar_sync(1 + g, 128);
+      trace_rec(pl.trace, 24 + g, E.gpass * 8 + 6, l == 0);
+      static_for<M>([&](auto I_) {
+        constexpr int i = I_;
+        const int ob = i % pl.NOB;
+        uint8_t* stg = ostage + (size_t)ob * pl.OSTRIDE;
+#pragma unroll
+        for (int j = 0; j < CPW / 4; ++j) {
+          float2 o[2] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
+          static_for<GP / 2>([&](auto Q_) {
+            constexpr int idx0 = PASS * GP + 2 * (int)Q_;
+            constexpr int tl0 = 2 * (int)Q_;
+            if constexpr (idx0 == 0) {
+              constexpr float c0 = T::AT(i, 0), c1 = T::AT(i, A - 1);
+#pragma unroll
+              for (int e = 0; e < 2; ++e) {
+                const float2 m0 = make_float2(mv[tl0][4 * j + 2 * e], mv[tl0][4 * j + 2 * e + 1]);
+                const float2 m1 = make_float2(mv[tl0 + 1][4 * j + 2 * e], mv[tl0 + 1][4 * j + 2 * e + 1]);
+                if constexpr (c0 != 0.f) o[e] = __ffma2_rn(make_float2(c0, c0), m0, o[e]);
+                if constexpr (c1 != 0.f) o[e] = __ffma2_rn(make_float2(c1, c1), m1, o[e]);
+              }
+            } else {
+              constexpr float ca = T::AT(i, point_of(idx0, A));
+              constexpr int src = (i % 2 == 0) ? tl0 : tl0 + 1;
+#pragma unroll
+              for (int e = 0; e < 2; ++e) {
+                const float2 ms = make_float2(mv[src][4 * j + 2 * e], mv[src][4 * j + 2 * e + 1]);
+                if constexpr (ca == 1.f) o[e] = __fadd2_rn(o[e], ms);
+                else if constexpr (ca != 0.f) o[e] = __ffma2_rn(make_float2(ca, ca), ms, o[e]);
+              }
+            }
+          });
+          if (live)
+            *reinterpret_cast<float4*>(stg + ((obase + (uint32_t)j * 16u) ^ oxor)) = make_float4(o[0].x, o[0].y, o[1].x, o[1].y);
+        }
+        fence_proxy_async_smem();
+        if (l == 0) bulk_wait_group_read_dyn(pl.NOB - 2);
+        named_bar_sync(1 + g, 128);
+        if (l == 0) {
+          const uint8_t* sbuf = ostage + (size_t)ob * pl.OSTRIDE;
+          const bool store = PASS == 0 && !E.split && !pl.ACCUM;
+          // one TMA op per run: columns tw m + i for the run's L tiles, rows [rb ROWS, +ROWS)
+          // (rows >= P and columns >= Q clipped by the TMA unit: the in-kernel boundary)
+#pragma unroll 1
+          for (int s = 0; s < nvalid;) {
+            const Strip st = strip_at(E.sg0 + s);
+            int L = 1;
+            while (s + L < nvalid && strip_at(E.sg0 + s + L).tw != 0) ++L;
+            const uint8_t* src = sbuf + s * Cfg::TSTRIDE;
+            const CUtensorMap* ymp = &ym.m[L - 1];
+            if (store) tma_store_4d(ymp, src, E.nb * NT + cbase, st.tw * M + i, st.rb * pl.ROWS, st.n);
+            else tma_reduce_add_4d(ymp, src, E.nb * NT + cbase, st.tw * M + i, st.rb * pl.ROWS, st.n);
+            s += L;
+          }
+          bulk_commit_group();
+        }
+        trace_rec(pl.trace, 24 + g, E.gpass * 8 + i, l == 0);
+      });
+      if (l == 0) bulk_wait_group_read<0>();
+      trace_rec(pl.trace, 24 + g, E.gpass * 8 + 7, l == 0);
+    };
+    auto epilogue = [&](const Epi& E) {
+      static_for<NPASS>([&](auto P_) { if ((int)P_ == E.pass) do_epilogue(P_, E); });
+    };
+
+    // Schedule: a pass's epilogue is deferred until after this warpgroup's FIRST chunk of the
+    // next pass (whose V slot frees as the pass's own MMAs complete), so while the MMAs drain
+    // the warpgroups already stage the next pass, and the next pass's first 4 chunks (one per
+    // warpgroup) are ready the moment every warpgroup has read its accumulators (d_empty).
+    // Only one chunk may run ahead: the next one would wait for MMAs that wait for d_empty.
+    int pc = 0;  // passes done
+    int gc = 0;  // global chunk counter (all passes of all items of this CTA)
+    bool pend = false;
+    Epi pe{0, 0, 0, 0, false};
+    for (int it = blockIdx.x; it < NITEMS; it += gridDim.x) {
+      const Item I = item_at(it);
+      const int sg0 = (I.ui / pl.NB) * 4, nb = I.ui % pl.NB;
+      for (int pass = I.pb; pass < I.pe; ++pass) {
+        const int gpass = pc++;
+        for (int cc = 0; cc < NCCL; ++cc, ++gc) {
+          if ((gc & (NWG - 1)) != g) continue;
+          static_for<NPASS>([&](auto P_) { if ((int)P_ == pass) do_chunk(P_, gc); });
+          if (pend) { epilogue(pe); pend = false; }
+        }
+        if (pend) { epilogue(pe); pend = false; }  // no chunk of this pass for this warpgroup
+        pe = Epi{gpass, pass, sg0, nb, I.split};
+        pend = true;
+      }
+    }
+    if (pend) epilogue(pe);
+  } else {
+    setmaxnreg_dec<56>();
+    if (warp == PROD_WARP) {
+      // ====================== input strip boxes (TMA) ======================
+      if (lane32 == 0) {
+        tma_prefetch_desc(&xmap);
+        for (int L = 0; L < 4; ++L) tma_prefetch_desc(&ym.m[L]);
+        asm volatile("griddepcontrol.wait;" ::: "memory");
+        int ist = 0, iph = 0, first = 1, gcp = 0;
+        for (int it = blockIdx.x; it < NITEMS; it += gridDim.x) {
+          const Item I = item_at(it);
+          const int sg0 = (I.ui / pl.NB) * 4;
+          Strip st[4];
+#pragma unroll
+          for (int s = 0; s < 4; ++s) st[s] = strip_at(min(sg0 + s, pl.NSTRIP - 1));
+          for (int pass = I.pb; pass < I.pe; ++pass) {
+            for (int cc = 0; cc < NCCL; ++cc, ++gcp) {
+              if (!first) mbar_wait(&in_empty[ist], iph ^ 1);
+              trace_rec(pl.trace, 31, gcp);
+              const int ca = chunk_of(I.ui, cc);
+              uint64_t* full = &in_full[gcp & 3];
+              mbar_expect_tx(full, 4u * SBOX);
+#pragma unroll
+              for (int s = 0; s < 4; ++s)
+                tma_load_4d(in_smem + ((size_t)ist * 4 + s) * SBOX, &xmap, full, ca * 8,
+                            st[s].tw * M - pl.pad_w, st[s].rb * pl.ROWS - pl.pad_h, st[s].n);
+              if (++ist == NIS) { ist = 0; iph ^= 1; first = 0; }
+            }
+          }
+        }
+      }
+      __syncwarp();
+    } else if (warp == UPROD_WARP) {
+      // ================= U (transformed filter) k-step ring =================
+      if (lane32 == 0) {
+        asm volatile("griddepcontrol.wait;" ::: "memory");
+        if (!I2CW_NO_TAGCHECK && blockIdx.x == 0) {
+          const UTag* tg = reinterpret_cast<const UTag*>(reinterpret_cast<const uint8_t*>(u) - kUTagBytes);
+          if (tg->magic != kUMagic || (int)tg->alpha != A || (int)tg->m != M || (int)tg->is_deconv != pl.is_deconv ||
+              (int)tg->C != pl.C || (int)tg->K != pl.K || (int)tg->R != pl.R || (int)tg->S != RW ||
+              (int)tg->NT != NT || (int)tg->halves != 1 || (int)tg->T != 1)
+            __trap();
+        }
+        const size_t kstride = (size_t)A * 2 * NT * 8;  // floats per k-step
+        int us = 0, uph = 0, first = 1;
+        for (int it = blockIdx.x; it < NITEMS; it += gridDim.x) {
+          const Item I = item_at(it);
+          const int nb = I.ui % pl.NB;
+          for (int pass = I.pb; pass < I.pe; ++pass) {
+            const float* src0 = u + u_offset(NT, A, nb, pl.NKS, 0, pass * GP, 0);
+            for (int cc = 0; cc < NCCL; ++cc) {
+              const int ca = chunk_of(I.ui, cc);
+              for (int fh = 0; fh < R; ++fh) {
+                if (!first) mbar_wait(&u_empty[us], uph ^ 1);
+                mbar_expect_tx(&u_full[us], UBYTES);
+                bulk_load(u_smem + (size_t)us * UBYTES, src0 + (size_t)(ca * R + fh) * kstride, UBYTES, &u_full[us]);
+                if (++us == NUS) { us = 0; uph ^= 1; first = 0; }
+              }
+            }
+          }
+        }
+      }
+      __syncwarp();
+    } else {
+      // ============================= MMA issuers =============================
+      const int iss = warp - ISS_WARP0;  // owns points tl = iss * PPI .. + PPI - 1
+      constexpr uint32_t idesc = idesc_tf32(128, NT);
+      const uint64_t bdesc0 = umma_desc_kmajor_noswizzle(smem_u32(u_smem), NT * 16, 128);
+      int us = 0, uph = 0, gc = 0, gpass = 0;
+      for (int it = blockIdx.x; it < NITEMS; it += gridDim.x) {
+        const Item I = item_at(it);
+        for (int pass = I.pb; pass < I.pe; ++pass, ++gpass) {
+          if (gpass > 0) {
+            mbar_wait(d_empty, (gpass - 1) & 1);
+            tc_fence_after();
+          }
+          for (int cc = 0; cc < NCCL; ++cc, ++gc) {
+            const int slot = gc & (NSLOT - 1);
+            trace_rec(pl.trace, 28, gc, iss == 0 && lane32 == 0);
+            mbar_wait(&st_full[slot], (gc / NSLOT) & 1);
+            trace_rec(pl.trace, 29, gc, iss == 0 && lane32 == 0);
+            tc_fence_after();
+            const uint32_t va = tbase + VCOL + (uint32_t)slot * GP * 16;
+            for (int fh = 0; fh < R; ++fh) {
+              mbar_wait(&u_full[us], uph);
+              tc_fence_after();
+              const uint64_t bk = bdesc0 + (uint64_t)((us * UBYTES) >> 4);
+#pragma unroll
+              for (int prod = 0; prod < 3; ++prod) {
+#pragma unroll
+                for (int pi = 0; pi < PPI; ++pi) {
+                  const int tl = iss * PPI + pi;
+                  const uint32_t a = va + tl * 16 + (prod == 0 ? 8 : 0);
+                  const uint64_t bd = bk + (uint64_t)(((tl * 2 + (prod == 1 ? 1 : 0)) * NT * 32) >> 4);
+                  const uint32_t acc = (cc > 0 || fh > 0 || prod > 0) ? 1u : 0u;
+                  mma_tf32_ts_warp(tbase + tl * NT, a, bd, idesc, acc);
+                }
+              }
+              mma_commit_warp(&u_empty[us]);
+              if (++us == NUS) { us = 0; uph ^= 1; }
+              if (fh + 1 < R) {  // next filter row: lane j takes lane j+1's input row
+#pragma unroll
+                for (int pi = 0; pi < PPI; ++pi) {
+                  const int tl = iss * PPI + pi;
+                  tmem_shift_up_warp(va + tl * 16);
+                  tmem_shift_up_warp(va + tl * 16 + 8);
+                }
+              }
+            }
+            mma_commit_warp(&st_empty[slot]);
+            trace_rec(pl.trace, 30, gc, iss == 0 && lane32 == 0);
+          }
+          mma_commit_warp(d_full);
+        }
+      }
+      __syncwarp();
+    }
+  }
+
+  tc_fence_before();
+  __syncthreads();
+  if (warp == ISS_WARP0) {
+    tc_fence_after();
+    tmem_dealloc(tbase, 512);
+  }
+}
+
+template <int M, int RW>
+static cudaError_t launch_strip_t(const CUtensorMap& xmap, const YMaps& ym, const Plan& pl, const float* u,
+                                  cudaStream_t stream) {
+  using Cfg = StripCfg<M, RW>;
+  auto kern = fused_strip_kernel<M, RW>;
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, pl.smem_bytes);
+  if (e != cudaSuccess) return e;
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(persistent_ctas(pl.NITEMS, 1));
+  cfg.blockDim = dim3(Cfg::NTHREADS);
+  cfg.dynamicSmemBytes = pl.smem_bytes;
+  cfg.stream = stream;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  e = cudaLaunchKernelEx(&cfg, kern, xmap, ym, pl, u);
+  if (e != cudaSuccess) return e;
+  return cudaGetLastError();
+}
+
+}  // namespace i2cw
