@@ -169,7 +169,9 @@ void plan_strip(Plan* plp, int nsm) {
   Plan& pl = *plp;
   static const int env = [] { const char* e = getenv("I2CW_STRIP"); return e ? atoi(e) : -1; }();
   pl.strip = 0;
-  if (env == 0 || pl.vol || pl.prec || pl.pair || pl.alpha != 8 || pl.NT != 64 || pl.R > 24) return;
+  if (env == 0 || pl.vol || pl.prec || pl.alpha != 8 || pl.NT != 64 || pl.R > 24) return;
+  // CTA pairs (M = 256, each SM streams half of U): I2CW_STRIP_PAIR=0/1 (default on)
+  static const int pair_env = [] { const char* e = getenv("I2CW_STRIP_PAIR"); return e ? atoi(e) : 1; }();
   const int rbmax = 33 - pl.R;
   const int pb = cdiv(pl.P, rbmax), rb = cdiv(pl.P, pb);
   const long long nstrip = (long long)pl.N * pb * pl.T_r;
@@ -180,7 +182,9 @@ void plan_strip(Plan* plp, int nsm) {
   const double util_strip = useful / ((double)sgroups * kMaxLanes);
   const double util_base = useful / ((double)pl.tile_blocks * kMaxLanes);
   if (env != 1 && util_strip < 0.85 * util_base) return;
-  constexpr int kUB = 4 * 2 * 64 * 32, kStage = 4 * 9 * 32 * 32;  // U k-step, 4 strip boxes (alpha = 8)
+  const int spair = pair_env != 0 && sgroups >= 2 ? 1 : 0;
+  const int kUB = 4 * 2 * (spair ? 32 : 64) * 32;  // this CTA's U k-step (alpha = 8, GP = 4)
+  constexpr int kStage = 4 * 9 * 32 * 32;           // 4 strip boxes (alpha = 8)
   const int osb = 4 * 2048, ostride = osb;  // 4 strips x 32 rows x 16 channels per output buffer
   // (U k-step slots, input stages, output buffers >= 2)
   static int kSD[][3] = {{8, 2, 2}, {6, 2, 2}, {5, 2, 2}, {4, 2, 2}, {3, 2, 2}, {2, 2, 2}};
@@ -193,12 +197,13 @@ void plan_strip(Plan* plp, int nsm) {
   (void)sd_env;
   int sel = -1, smem = 0;
   for (int d = 0; d < (int)(sizeof(kSD) / sizeof(kSD[0])); ++d) {
-    const int bar_bytes = 8 * (4 + kSD[d][1] + 10 + 2 * kSD[d][0]) + 16;
+    const int bar_bytes = 8 * (4 + kSD[d][1] + 10 + 2 * kSD[d][0]) + 32 + 4 * 4 * 16;  // + slot, epilogue op table
     smem = kSD[d][0] * kUB + kSD[d][1] * kStage + 4 * kSD[d][2] * ostride + bar_bytes;
     if (smem <= kSmemBudget) { sel = d; break; }
   }
   if (sel < 0) return;
   pl.strip = 1;
+  pl.pair = spair;
   pl.NSTRIP = (int)nstrip;
   pl.ROWS = rb;
   pl.PB = pb;
@@ -219,14 +224,15 @@ void plan_strip(Plan* plp, int nsm) {
   std::fill(pl.lane_row, pl.lane_row + kMaxLanes, 0);
   std::fill(pl.lane_in, pl.lane_in + kMaxLanes, 0);
   std::fill(pl.lane_tw, pl.lane_tw + kMaxLanes, 0);
-  const int units = sgroups * pl.NB;
-  const int tail = units % nsm;
+  const int units = (spair ? cdiv(sgroups, 2) : sgroups) * pl.NB;
+  const int G = spair ? std::max(1, nsm / 2) : nsm;
+  const int tail = units % G;
   const char* st = getenv("I2CW_SPLIT_TAIL");
   static const bool allsplit = [] { const char* e = getenv("I2CW_STRIP_ALLSPLIT"); return e && e[0] == '1'; }();
   if (pl.NPASS == 2 && allsplit) {  // experiments: every unit as two one-pass items
     pl.NFULL = 0;
     pl.NITEMS = 2 * units;
-  } else if (pl.NPASS == 2 && !(st && st[0] == '0') && tail > 0 && 2 * tail <= nsm) {
+  } else if (pl.NPASS == 2 && !(st && st[0] == '0') && tail > 0 && 2 * tail <= G) {
     pl.NFULL = units - tail;
     pl.NITEMS = pl.NFULL + 2 * tail;
   } else {
@@ -234,8 +240,9 @@ void plan_strip(Plan* plp, int nsm) {
   }
   const int item_ksteps = pl.NKS * (pl.NFULL > 0 ? pl.NPASS : 1);
   pl.KSL = 1;
-  if (pl.NKC == 1 && pl.NCC >= 2 && 2 * pl.NITEMS <= nsm)
-    pl.KSL = std::max(1, std::min({kslices_cap(), pl.NCC, nsm / std::max(1, pl.NITEMS), item_ksteps / 64}));
+  const int ctas = spair ? 2 * pl.NITEMS : pl.NITEMS;
+  if (pl.NKC == 1 && pl.NCC >= 2 && 2 * ctas <= nsm)
+    pl.KSL = std::max(1, std::min({kslices_cap(), pl.NCC, nsm / std::max(1, ctas), item_ksteps / 64}));
   if (pl.KSL > 1) pl.KSL = cdiv(pl.NCC, cdiv(pl.NCC, pl.KSL));
 }
 
@@ -857,6 +864,11 @@ int pretransformed_common(int is_deconv, int N, int H, int W, int C, int K, int 
   Plan pl;
   int rc = make_plan(N, H, W, C, K, R, S, pad_h, pad_w, is_deconv, &pl);
   if (rc != I2CW_OK) return rc;
+  if (pl.strip) {  // u has the base plan's layout (i2cw_filter_transform): keep the strip plan only if equal
+    Plan pb;
+    if ((rc = make_plan3(N, 1, H, W, C, K, 1, R, S, 0, pad_h, pad_w, is_deconv, 0, &pb, 2)) != I2CW_OK) return rc;
+    if (pb.pair != pl.pair) pl = pb;
+  }
   if ((rc = bind_device_of(x)) != I2CW_OK) return rc;
   auto matches = [&](const UTag& t) {
     return t.magic == kUMagic && (int)t.is_deconv == is_deconv && (int)t.C == C && (int)t.K == K && (int)t.R == R &&
@@ -979,15 +991,17 @@ int i2cw_deconv3d_ndhwc(int N, int D, int H, int W, int C, int K, int T, int R, 
 
 size_t i2cw_filter_bytes(int K, int C, int R, int S) {
   Plan pl;
-  // the filter-side plan fields do not depend on N, H, W or pad: plan a 1 x R x S map
-  if (make_plan(1, R, S, C, K, R, S, 0, 0, 0, &pl) != I2CW_OK) return 0;
+  // the filter-side plan fields do not depend on N, H, W or pad: plan a 1 x R x S map (base
+  // kernel layout; a call whose plan would use the strip kernel's CTA-pair layout instead runs
+  // the base kernel on a pre-transformed U, pretransformed_common)
+  if (make_plan3(1, 1, R, S, C, K, 1, R, S, 0, 0, 0, 0, 0, &pl, 2) != I2CW_OK) return 0;
   return kUTagBytes + u_data_bytes(pl);
 }
 
 int i2cw_filter_transform(int K, int C, int R, int S, int is_deconv, const float* w, void* u, i2cw_stream_t stream) {
   if (!w || !u || !aligned16(w) || !aligned16(u) || (is_deconv != 0 && is_deconv != 1)) return I2CW_EINVAL;
   Plan pl;
-  int rc = make_plan(1, R, S, C, K, R, S, 0, 0, 0, &pl);
+  int rc = make_plan3(1, 1, R, S, C, K, 1, R, S, 0, 0, 0, is_deconv, 0, &pl, 2);
   if (rc != I2CW_OK) return rc;
   if ((rc = bind_device_of(w)) != I2CW_OK) return rc;
   rc = transform_into(pl, is_deconv, w, u, (cudaStream_t)stream);

@@ -26,20 +26,29 @@
 
 namespace i2cw {
 
+template <bool PAIR>
 __device__ __forceinline__ void tmem_shift_up_warp(uint32_t taddr) {
   // PTX ".down" moves each row's 32-byte element to the row below in the matrix view, i.e. lane l
-  // receives lane l+1's value (measured, tools/shift_bench.cu); one elected lane issues
-  asm volatile(
-      "{\n\t.reg .pred e;\n\t"
-      "elect.sync _|e, 0xffffffff;\n\t"
-      "@e tcgen05.shift.cta_group::1.down [%0];\n\t}" ::"r"(taddr)
-      : "memory");
+  // receives lane l+1's value (measured, tools/shift_bench.cu); one elected lane issues. The
+  // cta_group::2 form shifts both CTAs of a pair (tools/shift2_bench.cu).
+  if constexpr (PAIR)
+    asm volatile(
+        "{\n\t.reg .pred e;\n\t"
+        "elect.sync _|e, 0xffffffff;\n\t"
+        "@e tcgen05.shift.cta_group::2.down [%0];\n\t}" ::"r"(taddr)
+        : "memory");
+  else
+    asm volatile(
+        "{\n\t.reg .pred e;\n\t"
+        "elect.sync _|e, 0xffffffff;\n\t"
+        "@e tcgen05.shift.cta_group::1.down [%0];\n\t}" ::"r"(taddr)
+        : "memory");
 }
 
 constexpr int kStripLanes = 32;  // input rows per strip box (one TMEM subpartition)
 struct alignas(64) YMaps { CUtensorMap m[4]; };  // y store maps for runs of 1..4 strips
 
-template <int M, int RW>
+template <int M, int RW, bool PAIR>
 struct StripCfg {
   using T = Wino<M, RW>;
   static constexpr int A = T::alpha;
@@ -51,7 +60,8 @@ struct StripCfg {
   static constexpr int NISS = niss_for(GP);
   static constexpr int PPI = GP / NISS;
   static constexpr int VCOL = GP * NT;
-  static constexpr int UBYTES = GP * 2 * NT * 32;                // one k-step of U (GP points, hi + lo)
+  static constexpr int BROWS = PAIR ? NT / 2 : NT;               // B rows (output channels) held per CTA
+  static constexpr int UBYTES = GP * 2 * BROWS * 32;             // one k-step of this CTA's U (GP points, hi + lo)
   // one strip's input box: 8 ch x (A + 1) cols x 32 rows, smem image [row][col][8 ch] with the TMA
   // 32B swizzle; the 9th column makes the row stride 288 B, so 8 consecutive rows read 8 distinct
   // 16-byte bank groups (a 256-byte stride with any swizzle leaves 2-way conflicts)
@@ -71,12 +81,19 @@ struct StripCfg {
 // per output column (a box may not start at a negative column, so a run that starts inside the
 // unit needs its exact length); swizzle 64B for L = 3, else 128B (conflict-free or 2-way
 // staging writes).
-template <int M, int RW>
-__global__ void __launch_bounds__(StripCfg<M, RW>::NTHREADS, 1)
+// PAIR: a cluster of 2 CTAs on an SM pair, tcgen05.mma.cta_group::2 with M = 256 (each CTA's 4
+// strips) and N = 64; each CTA stages only its half of the U rows (halving the per-SM filter
+// stream from L2 and the B-operand reads from shared memory). The leader (rank 0) issues all
+// MMAs and shifts; the peer's warps arrive remotely on the leader's V / accumulator barriers and
+// a peer thread forwards "my U half landed"; commits are multicast to both CTAs.
+template <int M, int RW, bool PAIR>
+__global__ void __launch_bounds__(StripCfg<M, RW, PAIR>::NTHREADS, 1)
     fused_strip_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__ YMaps ym,
                        const __grid_constant__ Plan pl, const float* __restrict__ u) {
-  using Cfg = StripCfg<M, RW>;
+  using Cfg = StripCfg<M, RW, PAIR>;
   using T = typename Cfg::T;
+  constexpr int BROWS = Cfg::BROWS;
+  const uint32_t rank = PAIR ? cluster_ctarank() : 0u;  // 0 = MMA leader
   constexpr int A = Cfg::A, GP = Cfg::GP, NPASS = Cfg::NPASS, NWG = Cfg::NWG, NSLOT = Cfg::NSLOT;
   constexpr int NISS = Cfg::NISS, PPI = Cfg::PPI, VCOL = Cfg::VCOL, NT = Cfg::NT;
   constexpr uint32_t UBYTES = Cfg::UBYTES, SBOX = Cfg::SBOX;
@@ -102,9 +119,15 @@ __global__ void __launch_bounds__(StripCfg<M, RW>::NTHREADS, 1)
   uint64_t* u_full = d_empty + 1;        // [NUS]
   uint64_t* u_empty = u_full + NUS;      // [NUS]
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(u_empty + NUS);
+  // [NWG][4] store ops of the pending epilogue (16-byte aligned, after the TMEM slot word)
+  int4* epi_ops = reinterpret_cast<int4*>((reinterpret_cast<uintptr_t>(u_empty + NUS + 1) + 15) & ~uintptr_t(15));
 
   const int warp = threadIdx.x / 32, lane32 = threadIdx.x % 32;
   const int NITEMS = pl.NITEMS;
+  // persistent schedule over work units (CTA pairs share a unit: strip groups 2k, 2k + 1)
+  const int unit0 = PAIR ? (int)(blockIdx.x >> 1) : (int)blockIdx.x;
+  const int ustride = PAIR ? (int)(gridDim.x >> 1) : (int)gridDim.x;
+  auto sg0_of = [&](int ui) { return ((PAIR ? 2 * (ui / pl.NB) + (int)rank : ui / pl.NB)) * 4; };
   struct Item { int ui, pb, pe; bool split; };
   auto item_at = [&](int it) {
     Item I;
@@ -132,17 +155,26 @@ __global__ void __launch_bounds__(StripCfg<M, RW>::NTHREADS, 1)
   if (threadIdx.x == 0) {
     for (int i = 0; i < 4; ++i) mbar_init(&in_full[i], 1);
     for (int i = 0; i < NIS; ++i) mbar_init(&in_empty[i], 4);
-    for (int i = 0; i < NSLOT; ++i) { mbar_init(&st_full[i], 4); mbar_init(&st_empty[i], NISS); }
-    for (int i = 0; i < NUS; ++i) { mbar_init(&u_full[i], 1); mbar_init(&u_empty[i], NISS); }
+    const int lead2 = PAIR && rank == 0 ? 2 : 1;  // the pair leader also counts the peer's arrivals
+    for (int i = 0; i < NSLOT; ++i) { mbar_init(&st_full[i], 4 * lead2); mbar_init(&st_empty[i], NISS); }
+    for (int i = 0; i < NUS; ++i) { mbar_init(&u_full[i], lead2); mbar_init(&u_empty[i], NISS); }
     mbar_init(d_full, NISS);
-    mbar_init(d_empty, NWG * 4);
+    mbar_init(d_empty, NWG * 4 * lead2);
     fence_mbar_init();
   }
-  if (warp == ISS_WARP0) { tmem_alloc(tmem_slot, 512); tmem_relinquish(); }
+  if (warp == ISS_WARP0) {
+    if constexpr (PAIR) { tmem_alloc2(tmem_slot, 512); tmem_relinquish2(); }
+    else { tmem_alloc(tmem_slot, 512); tmem_relinquish(); }
+  }
   tc_fence_before();
-  __syncthreads();
+  if constexpr (PAIR) cluster_sync_all();
+  else __syncthreads();
   tc_fence_after();
   const uint32_t tbase = *tmem_slot;
+#if I2CW_TRACE
+  // per-CTA start / end (globaltimer ns) after the 32 x 512 x 2 timeline records
+  if (pl.trace != nullptr && threadIdx.x == 0) pl.trace[2 * 32 * 512 + 2 * blockIdx.x] = globaltimer();
+#endif
 
   if (warp < NWG * 4) {
     setmaxnreg_inc<104>();
@@ -156,6 +188,7 @@ __global__ void __launch_bounds__(StripCfg<M, RW>::NTHREADS, 1)
     const uint32_t rofs = (uint32_t)jr * (Cfg::WCOL * 32);  // this lane's row in the box
     const bool out_row = jr < pl.ROWS;  // output row of the strip (else: halo input row only)
     uint8_t* ostage = o_smem + (size_t)g * pl.NOB * pl.OSTRIDE;
+    const uint32_t st_full_lead = PAIR ? mapa_shared(st_full, 0) : 0u, d_empty_lead = PAIR ? mapa_shared(d_empty, 0) : 0u;
     // ---- one chunk of V (this warpgroup's chunk gc of a pass with point group PASS) ----
     auto do_chunk = [&](auto PASS_, int gc) {
       constexpr int PASS = PASS_;
@@ -210,7 +243,7 @@ __global__ void __launch_bounds__(StripCfg<M, RW>::NTHREADS, 1)
       }
       trace_rec(pl.trace, 8 + g, gc / NWG, l == 0);
       const int use = gc / NSLOT;
-      if (use > 0) mbar_wait(&st_empty[g], (use - 1) & 1);
+      if (use > 0) mbar_wait_tc<PAIR>(&st_empty[g], (use - 1) & 1);
       trace_rec(pl.trace, 12 + g, gc / NWG, l == 0);
       tc_fence_after();
 #pragma unroll
@@ -228,7 +261,10 @@ __global__ void __launch_bounds__(StripCfg<M, RW>::NTHREADS, 1)
       tmem_wait_st();
       tc_fence_before();
       __syncwarp();
-      if (lane32 == 0) mbar_arrive(&st_full[g]);
+      if (lane32 == 0) {
+        if (PAIR && rank == 1) mbar_arrive_remote(st_full_lead + 8u * (uint32_t)g);
+        else mbar_arrive(&st_full[g]);
+      }
       trace_rec(pl.trace, 16 + g, gc / NWG, l == 0);
     };
 
@@ -239,18 +275,40 @@ __global__ void __launch_bounds__(StripCfg<M, RW>::NTHREADS, 1)
       // runs of the unit: strips with the same (n, rb) (a run starts at s = 0 or where tw = 0).
       // This warp's strip sub is tile t = sub - r0 of the run [r0, r0 + rl); the run's staging
       // region starts at r0 * TSTRIDE and holds [row][rl tiles][16 ch] (the box image of map rl)
-      const int nvalid = min(4, pl.NSTRIP - E.sg0);
+      const int nvalid = max(0, min(4, pl.NSTRIP - E.sg0));  // 0: a pair's idle half
       int r0 = 0, rl = 1;
       for (int s = 1; s <= sub; ++s)
         if (s < nvalid && strip_at(E.sg0 + s).tw == 0) r0 = s;
       while (r0 + rl < nvalid && strip_at(E.sg0 + r0 + rl).tw != 0) ++rl;
+      // a run of 4 is stored as 3 + 1 tiles: with 64-byte staging rows the 4-tile box image puts
+      // 8 consecutive rows of one tile in 2 bank groups (4-way conflicts, measured), 3 and 1 tiles
+      // are conflict-free
+      if (rl == 4) { if (sub < r0 + 3) rl = 3; else { r0 += 3; rl = 1; } }
       // staging offset of this lane's row (bytes, before the swizzle) and the swizzle of map rl
       // (64B for rl = 3: chunk bits [5:4] ^= [8:7]; else 128B: [6:4] ^= [9:7])
       const uint32_t obase = (uint32_t)(r0 * Cfg::TSTRIDE + (jr * rl + (sub - r0)) * 64);
       const uint32_t oxor = ((obase >> 7) & 3u) << 4;
       const bool live = out_row && sub < nvalid;
+      // the unit's TMA store ops (one per run piece), computed once for all columns by thread 0
+      // into shared memory: {staging start s | (length - 1) << 8, column tw m, row, image}
+      int4* ops = epi_ops + g * 4;
+      int nops = 0;
+      if (l == 0) {
+        int cur_s = 0, cur_L = 0;
+        for (int s = 0; s < nvalid; ++s) {
+          const Strip st = strip_at(E.sg0 + s);
+          if (s == 0 || st.tw == 0 || cur_L == 3) {
+            ops[nops] = make_int4(s, st.tw * M, st.rb * pl.ROWS, st.n);
+            cur_s = s; cur_L = 1;
+            ++nops;
+          } else {
+            ++cur_L;
+          }
+          ops[nops - 1].x = cur_s | ((cur_L - 1) << 8);
+        }
+      }
       trace_rec(pl.trace, 20 + g, 2 * E.gpass, l == 0);
-      mbar_wait(d_full, E.gpass & 1);
+      mbar_wait_tc<PAIR>(d_full, E.gpass & 1);
       trace_rec(pl.trace, 20 + g, 2 * E.gpass + 1, l == 0);
       tc_fence_after();
       const int cbase = g * CPW;
@@ -260,7 +318,11 @@ __global__ void __launch_bounds__(StripCfg<M, RW>::NTHREADS, 1)
       tmem_wait_ld();
       tc_fence_before();
       __syncwarp();
-      if (lane32 == 0) mbar_arrive(d_empty);  // accumulators read: the next pass's MMAs may start
+      if (lane32 == 0) {  // accumulators read: the next pass's MMAs may start
+        if (PAIR && rank == 1) mbar_arrive_remote(d_empty_lead);
+        else mbar_arrive(d_empty);
+      }
+      if (ABL(4)) return;  // DEBUG timing ablation: no output transform / y
       static_for<GP / 2>([&](auto Q_) {  // pair (a, a+1): AT[i][a+1] = (-1)^i AT[i][a]
         constexpr int idx0 = PASS * GP + 2 * (int)Q_;
         constexpr int tl0 = 2 * (int)Q_;
@@ -323,15 +385,13 @@ __global__ void __launch_bounds__(StripCfg<M, RW>::NTHREADS, 1)
           // one TMA op per run: columns tw m + i for the run's L tiles, rows [rb ROWS, +ROWS)
           // (rows >= P and columns >= Q clipped by the TMA unit: the in-kernel boundary)
 #pragma unroll 1
-          for (int s = 0; s < nvalid;) {
-            const Strip st = strip_at(E.sg0 + s);
-            int L = 1;
-            while (s + L < nvalid && strip_at(E.sg0 + s + L).tw != 0) ++L;
-            const uint8_t* src = sbuf + s * Cfg::TSTRIDE;
-            const CUtensorMap* ymp = &ym.m[L - 1];
-            if (store) tma_store_4d(ymp, src, E.nb * NT + cbase, st.tw * M + i, st.rb * pl.ROWS, st.n);
-            else tma_reduce_add_4d(ymp, src, E.nb * NT + cbase, st.tw * M + i, st.rb * pl.ROWS, st.n);
-            s += L;
+          for (int k = 0; k < nops; ++k) {
+            if (ABL(32)) break;  // DEBUG timing ablation: no y writes
+            const int4 op = ops[k];
+            const uint8_t* src = sbuf + (op.x & 0xff) * Cfg::TSTRIDE;
+            const CUtensorMap* ymp = &ym.m[op.x >> 8];
+            if (store) tma_store_4d(ymp, src, E.nb * NT + cbase, op.y + i, op.z, op.w);
+            else tma_reduce_add_4d(ymp, src, E.nb * NT + cbase, op.y + i, op.z, op.w);
           }
           bulk_commit_group();
         }
@@ -353,9 +413,9 @@ __global__ void __launch_bounds__(StripCfg<M, RW>::NTHREADS, 1)
     int gc = 0;  // global chunk counter (all passes of all items of this CTA)
     bool pend = false;
     Epi pe{0, 0, 0, 0, false};
-    for (int it = blockIdx.x; it < NITEMS; it += gridDim.x) {
+    for (int it = unit0; it < NITEMS; it += ustride) {
       const Item I = item_at(it);
-      const int sg0 = (I.ui / pl.NB) * 4, nb = I.ui % pl.NB;
+      const int sg0 = sg0_of(I.ui), nb = I.ui % pl.NB;
       for (int pass = I.pb; pass < I.pe; ++pass) {
         const int gpass = pc++;
         for (int cc = 0; cc < NCCL; ++cc, ++gc) {
@@ -378,9 +438,9 @@ __global__ void __launch_bounds__(StripCfg<M, RW>::NTHREADS, 1)
         for (int L = 0; L < 4; ++L) tma_prefetch_desc(&ym.m[L]);
         asm volatile("griddepcontrol.wait;" ::: "memory");
         int ist = 0, iph = 0, first = 1, gcp = 0;
-        for (int it = blockIdx.x; it < NITEMS; it += gridDim.x) {
+        for (int it = unit0; it < NITEMS; it += ustride) {
           const Item I = item_at(it);
-          const int sg0 = (I.ui / pl.NB) * 4;
+          const int sg0 = sg0_of(I.ui);
           Strip st[4];
 #pragma unroll
           for (int s = 0; s < 4; ++s) st[s] = strip_at(min(sg0 + s, pl.NSTRIP - 1));
@@ -409,20 +469,22 @@ __global__ void __launch_bounds__(StripCfg<M, RW>::NTHREADS, 1)
           const UTag* tg = reinterpret_cast<const UTag*>(reinterpret_cast<const uint8_t*>(u) - kUTagBytes);
           if (tg->magic != kUMagic || (int)tg->alpha != A || (int)tg->m != M || (int)tg->is_deconv != pl.is_deconv ||
               (int)tg->C != pl.C || (int)tg->K != pl.K || (int)tg->R != pl.R || (int)tg->S != RW ||
-              (int)tg->NT != NT || (int)tg->halves != 1 || (int)tg->T != 1)
+              (int)tg->NT != NT || (int)tg->halves != (PAIR ? 2 : 1) || (int)tg->T != 1)
             __trap();
         }
         const size_t kstride = (size_t)A * 2 * NT * 8;  // floats per k-step
         int us = 0, uph = 0, first = 1;
-        for (int it = blockIdx.x; it < NITEMS; it += gridDim.x) {
+        for (int it = unit0; it < NITEMS; it += ustride) {
           const Item I = item_at(it);
           const int nb = I.ui % pl.NB;
           for (int pass = I.pb; pass < I.pe; ++pass) {
-            const float* src0 = u + u_offset(NT, A, nb, pl.NKS, 0, pass * GP, 0);
+            // this CTA's B rows of the pass's GP points, hi + lo, contiguous (pair: its N half)
+            const float* src0 = u + (PAIR ? u_offset_pair(NT, A, nb, pl.NKS, 0, (int)rank, pass * GP)
+                                          : u_offset(NT, A, nb, pl.NKS, 0, pass * GP, 0));
             for (int cc = 0; cc < NCCL; ++cc) {
               const int ca = chunk_of(I.ui, cc);
               for (int fh = 0; fh < R; ++fh) {
-                if (!first) mbar_wait(&u_empty[us], uph ^ 1);
+                if (!first) mbar_wait_tc<PAIR>(&u_empty[us], uph ^ 1);
                 mbar_expect_tx(&u_full[us], UBYTES);
                 bulk_load(u_smem + (size_t)us * UBYTES, src0 + (size_t)(ca * R + fh) * kstride, UBYTES, &u_full[us]);
                 if (++us == NUS) { us = 0; uph ^= 1; first = 0; }
@@ -435,20 +497,36 @@ __global__ void __launch_bounds__(StripCfg<M, RW>::NTHREADS, 1)
     } else {
       // ============================= MMA issuers =============================
       const int iss = warp - ISS_WARP0;  // owns points tl = iss * PPI .. + PPI - 1
-      constexpr uint32_t idesc = idesc_tf32(128, NT);
-      const uint64_t bdesc0 = umma_desc_kmajor_noswizzle(smem_u32(u_smem), NT * 16, 128);
+      constexpr uint32_t idesc = idesc_tf32(PAIR ? 256 : 128, NT);
+      const uint64_t bdesc0 = umma_desc_kmajor_noswizzle(smem_u32(u_smem), BROWS * 16, 128);
       int us = 0, uph = 0, gc = 0, gpass = 0;
-      for (int it = blockIdx.x; it < NITEMS; it += gridDim.x) {
+      if (PAIR && rank == 1) {
+        // pair peer: forward "my U half landed" to the leader's U slot (off the critical path:
+        // the U ring runs ahead)
+        if (iss == 0 && lane32 == 0) {
+          const uint32_t lead_ufull = mapa_shared(u_full, 0);
+          for (int it = unit0; it < NITEMS; it += ustride) {
+            const Item I = item_at(it);
+            for (int pass = I.pb; pass < I.pe; ++pass)
+              for (int k = 0; k < NCCL * R; ++k) {
+                mbar_wait_tc<PAIR>(&u_full[us], uph);
+                mbar_arrive_remote(lead_ufull + 8u * (uint32_t)us);
+                if (++us == NUS) { us = 0; uph ^= 1; }
+              }
+          }
+        }
+      } else
+      for (int it = unit0; it < NITEMS; it += ustride) {
         const Item I = item_at(it);
         for (int pass = I.pb; pass < I.pe; ++pass, ++gpass) {
           if (gpass > 0) {
-            mbar_wait(d_empty, (gpass - 1) & 1);
+            mbar_wait_tc<PAIR>(d_empty, (gpass - 1) & 1);
             tc_fence_after();
           }
           for (int cc = 0; cc < NCCL; ++cc, ++gc) {
             const int slot = gc & (NSLOT - 1);
             trace_rec(pl.trace, 28, gc, iss == 0 && lane32 == 0);
-            mbar_wait(&st_full[slot], (gc / NSLOT) & 1);
+            mbar_wait_tc<PAIR>(&st_full[slot], (gc / NSLOT) & 1);
             trace_rec(pl.trace, 29, gc, iss == 0 && lane32 == 0);
             tc_fence_after();
             const uint32_t va = tbase + VCOL + (uint32_t)slot * GP * 16;
@@ -456,32 +534,38 @@ __global__ void __launch_bounds__(StripCfg<M, RW>::NTHREADS, 1)
               mbar_wait(&u_full[us], uph);
               tc_fence_after();
               const uint64_t bk = bdesc0 + (uint64_t)((us * UBYTES) >> 4);
+              if (!ABL(2)) {
 #pragma unroll
               for (int prod = 0; prod < 3; ++prod) {
 #pragma unroll
                 for (int pi = 0; pi < PPI; ++pi) {
                   const int tl = iss * PPI + pi;
                   const uint32_t a = va + tl * 16 + (prod == 0 ? 8 : 0);
-                  const uint64_t bd = bk + (uint64_t)(((tl * 2 + (prod == 1 ? 1 : 0)) * NT * 32) >> 4);
+                  const uint64_t bd = bk + (uint64_t)(((tl * 2 + (prod == 1 ? 1 : 0)) * BROWS * 32) >> 4);
                   const uint32_t acc = (cc > 0 || fh > 0 || prod > 0) ? 1u : 0u;
-                  mma_tf32_ts_warp(tbase + tl * NT, a, bd, idesc, acc);
+                  if constexpr (PAIR) mma2_tf32_ts_warp(tbase + tl * NT, a, bd, idesc, acc);
+                  else mma_tf32_ts_warp(tbase + tl * NT, a, bd, idesc, acc);
                 }
               }
-              mma_commit_warp(&u_empty[us]);
+              }
+              if constexpr (PAIR) mma_commit2_warp(&u_empty[us]);
+              else mma_commit_warp(&u_empty[us]);
               if (++us == NUS) { us = 0; uph ^= 1; }
-              if (fh + 1 < R) {  // next filter row: lane j takes lane j+1's input row
+              if (fh + 1 < R && !ABL(2)) {  // next filter row: lane j takes lane j+1's input row
 #pragma unroll
                 for (int pi = 0; pi < PPI; ++pi) {
                   const int tl = iss * PPI + pi;
-                  tmem_shift_up_warp(va + tl * 16);
-                  tmem_shift_up_warp(va + tl * 16 + 8);
+                  tmem_shift_up_warp<PAIR>(va + tl * 16);
+                  tmem_shift_up_warp<PAIR>(va + tl * 16 + 8);
                 }
               }
             }
-            mma_commit_warp(&st_empty[slot]);
+            if constexpr (PAIR) mma_commit2_warp(&st_empty[slot]);
+            else mma_commit_warp(&st_empty[slot]);
             trace_rec(pl.trace, 30, gc, iss == 0 && lane32 == 0);
           }
-          mma_commit_warp(d_full);
+          if constexpr (PAIR) mma_commit2_warp(d_full);
+          else mma_commit_warp(d_full);
         }
       }
       __syncwarp();
@@ -489,30 +573,44 @@ __global__ void __launch_bounds__(StripCfg<M, RW>::NTHREADS, 1)
   }
 
   tc_fence_before();
-  __syncthreads();
+  if constexpr (PAIR) cluster_sync_all();
+  else __syncthreads();
+#if I2CW_TRACE
+  if (pl.trace != nullptr && threadIdx.x == 0) pl.trace[2 * 32 * 512 + 2 * blockIdx.x + 1] = globaltimer();
+#endif
   if (warp == ISS_WARP0) {
     tc_fence_after();
-    tmem_dealloc(tbase, 512);
+    if constexpr (PAIR) tmem_dealloc2(tbase, 512);
+    else tmem_dealloc(tbase, 512);
   }
 }
 
-template <int M, int RW>
+template <int M, int RW, bool PAIR>
 static cudaError_t launch_strip_t(const CUtensorMap& xmap, const YMaps& ym, const Plan& pl, const float* u,
                                   cudaStream_t stream) {
-  using Cfg = StripCfg<M, RW>;
-  auto kern = fused_strip_kernel<M, RW>;
+  using Cfg = StripCfg<M, RW, PAIR>;
+  auto kern = fused_strip_kernel<M, RW, PAIR>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, pl.smem_bytes);
   if (e != cudaSuccess) return e;
   cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = dim3(persistent_ctas(pl.NITEMS, 1));
+  cfg.gridDim = dim3(persistent_ctas(pl.NITEMS, PAIR ? 2 : 1));
   cfg.blockDim = dim3(Cfg::NTHREADS);
   cfg.dynamicSmemBytes = pl.smem_bytes;
   cfg.stream = stream;
-  cudaLaunchAttribute attr[1];
-  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cudaLaunchAttribute attr[2];
+  int na = 0;
+  if constexpr (PAIR) {
+    attr[na].id = cudaLaunchAttributeClusterDimension;
+    attr[na].val.clusterDim.x = 2;
+    attr[na].val.clusterDim.y = 1;
+    attr[na].val.clusterDim.z = 1;
+    ++na;
+  }
+  attr[na].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[na].val.programmaticStreamSerializationAllowed = 1;
+  ++na;
   cfg.attrs = attr;
-  cfg.numAttrs = 1;
+  cfg.numAttrs = na;
   e = cudaLaunchKernelEx(&cfg, kern, xmap, ym, pl, u);
   if (e != cudaSuccess) return e;
   return cudaGetLastError();

@@ -18,18 +18,27 @@ for name in sys.argv[1:] or ["cfg2"]:
     x = torch.rand((N, H, W, C), device="cuda"); w = torch.rand((K, R, S, C), device="cuda")
     P, Q = H + 2 * ph - R + 1, W + 2 * pw - S + 1
     y = torch.empty((N, P, Q, K), device="cuda")
-    tr = torch.zeros(2 * 32 * 512, dtype=torch.int64, device="cuda")
+    tr = torch.zeros(2 * 32 * 512 + 2 * 160, dtype=torch.int64, device="cuda")
     for _ in range(3):
         tr.zero_()
         rc = L.i2cw_debug_trace(0, N, H, W, C, K, R, S, ph, pw, x.data_ptr(), w.data_ptr(), y.data_ptr(), tr.data_ptr(),
                                 torch.cuda.current_stream().cuda_stream)
         assert rc == 0
     torch.cuda.synchronize()
-    T = tr.cpu().numpy().reshape(2, 32, 512).astype(np.int64)[0]
+    TT = tr.cpu().numpy().astype(np.int64)
+    cta = TT[2 * 32 * 512:].reshape(-1, 2)
+    cta = cta[cta[:, 0] > 0]
+    T = TT[:2 * 32 * 512].reshape(2, 32, 512)[0]
     t0 = T[T > 0].min()
     T = np.where(T > 0, T - t0, -1)
     v = lambda k: T[k][T[k] >= 0]
     pl = i2cw.debug_plan(kind, N, H, W, C, K, R, S, ph, pw)
+    if len(cta):
+        t0c = cta[:, 0].min()
+        st, en = (cta[:, 0] - t0c) / 1e3, (cta[:, 1] - t0c) / 1e3
+        print(f"per-CTA (us): start max {st.max():.1f}; end min {en.min():.1f} median {np.median(en):.1f} max {en.max():.1f}; "
+              f"kernel span {en.max():.1f}")
+        print("  end times sorted (every 8th):", np.round(np.sort(en)[::8], 1).tolist())
     print(f"== {name}: strip {pl['strip']} NUS {pl['NUS']} NIS {pl['NIS']} NOB {pl['NOB']} NITEMS {pl['NITEMS']} "
           f"tile_blocks {pl['tile_blocks']}")
     for g in range(4):
