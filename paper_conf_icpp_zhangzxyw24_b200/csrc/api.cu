@@ -80,10 +80,16 @@ int alpha_env() {
   static const int v = [] { const char* e = getenv("I2CW_ALPHA"); return e ? atoi(e) : 0; }();
   return v;
 }
+bool strip_enabled() {
+  static const bool on = [] { const char* e = getenv("I2CW_STRIP"); return !(e && e[0] == '0'); }();
+  return on;
+}
 bool choose(int S, int C, Choice* c) {
   if (alpha16_override() && S >= 7 && S <= 9) { *c = {17 - S, 16, 1}; return true; }
   if (S == 2 || S == 3) {
-    const bool a4 = alpha_env() == 4 || (alpha_env() != 8 && (S == 2 || C >= 256));
+    // r = 3 at C >= 256: the strip kernel (alpha = 8 only) with F(6,3) beats the base kernel's best
+    // alpha = 4 plan by ~21% on cfg5b c256 / c512 (profiles/r02_strip_sweep.txt)
+    const bool a4 = alpha_env() == 4 || (alpha_env() != 8 && (S == 2 || (C >= 256 && !strip_enabled())));
     *c = a4 ? Choice{5 - S, 4, 0} : Choice{9 - S, 8, 0};
     return true;
   }
@@ -165,7 +171,7 @@ int num_sms() {
 // 4 consecutive strips in (n, row block, tw) order. Used for the 2D 3xTF32 alpha = 8 single-CTA
 // plans (the U layout of the pair plans differs) when its lane use is not much worse than the
 // base block shape's. I2CW_STRIP=0/1 disables / forces it (experiments).
-void plan_strip(Plan* plp, int nsm) {
+void plan_strip(Plan* plp, int nsm, bool nopair) {
   Plan& pl = *plp;
   static const int env = [] { const char* e = getenv("I2CW_STRIP"); return e ? atoi(e) : -1; }();
   pl.strip = 0;
@@ -181,8 +187,10 @@ void plan_strip(Plan* plp, int nsm) {
   const double useful = (double)pl.N * pl.P * pl.T_r;
   const double util_strip = useful / ((double)sgroups * kMaxLanes);
   const double util_base = useful / ((double)pl.tile_blocks * kMaxLanes);
-  if (env != 1 && util_strip < 0.85 * util_base) return;
-  const int spair = pair_env != 0 && sgroups >= 2 ? 1 : 0;
+  // measured on B200 (profiles/r02_strip_sweep.txt): the strip kernel wins from a lane-use ratio
+  // of 0.8 (cfg5a +2.5%, cfg2 +10%, cfg5b +14..21%) and loses below 0.7 (P = 32 images: cfg3)
+  if (env != 1 && util_strip < 0.75 * util_base) return;
+  const int spair = pair_env != 0 && !nopair && sgroups >= 2 ? 1 : 0;
   const int kUB = 4 * 2 * (spair ? 32 : 64) * 32;  // this CTA's U k-step (alpha = 8, GP = 4)
   constexpr int kStage = 4 * 9 * 32 * 32;           // 4 strip boxes (alpha = 8)
   const int osb = 4 * 2048, ostride = osb;  // 4 strips x 32 rows x 16 channels per output buffer
@@ -256,7 +264,7 @@ int make_plan_uncached(int N, int D, int H, int W, int C, int K, int T, int R, i
       pad_h < 0 || pad_w < 0)
     return I2CW_EINVAL;
   if (!vol && (D != 1 || T != 1 || pad_d != 0)) return I2CW_EINVAL;
-  const int nostrip = prec & 2;
+  const int nostrip = prec & 2, strip_nopair = prec & 4;
   prec &= 1;
   if (prec && vol) return I2CW_EUNSUPPORTED;  // 1xTF32 kernels: 2D only
   Choice ch;
@@ -448,7 +456,9 @@ int make_plan_uncached(int N, int D, int H, int W, int C, int K, int T, int R, i
       pl.KSL = std::max(1, std::min({kslices_cap(), pl.NCC, nsm / std::max(1, ctas), item_ksteps / 64}));
     if (pl.KSL > 1) pl.KSL = cdiv(pl.NCC, cdiv(pl.NCC, pl.KSL));  // no empty slice
   }
-  if (!nostrip) plan_strip(&pl, nsm);  // prec bit 1: base plan only (the SIMT stepping stone)
+  // prec bit 1: base plan only (the SIMT stepping stone, filter-only plans); bit 2: no CTA pairs
+  // in the strip plan (a pre-transformed U in the single-CTA layout)
+  if (!nostrip) plan_strip(&pl, nsm, strip_nopair != 0);
   *out = pl;
   return I2CW_OK;
 }
@@ -864,10 +874,12 @@ int pretransformed_common(int is_deconv, int N, int H, int W, int C, int K, int 
   Plan pl;
   int rc = make_plan(N, H, W, C, K, R, S, pad_h, pad_w, is_deconv, &pl);
   if (rc != I2CW_OK) return rc;
-  if (pl.strip) {  // u has the base plan's layout (i2cw_filter_transform): keep the strip plan only if equal
+  if (pl.strip && pl.pair) {  // u has the filter-only (base) plan's layout (i2cw_filter_transform)
     Plan pb;
     if ((rc = make_plan3(N, 1, H, W, C, K, 1, R, S, 0, pad_h, pad_w, is_deconv, 0, &pb, 2)) != I2CW_OK) return rc;
-    if (pb.pair != pl.pair) pl = pb;
+    // the single-CTA strip kernel reads that layout and sums in the same order (bitwise equal)
+    if (!pb.pair && (rc = make_plan3(N, 1, H, W, C, K, 1, R, S, 0, pad_h, pad_w, is_deconv, 0, &pl, 4)) != I2CW_OK)
+      return rc;
   }
   if ((rc = bind_device_of(x)) != I2CW_OK) return rc;
   auto matches = [&](const UTag& t) {

@@ -145,9 +145,12 @@ __global__ void __launch_bounds__(StripCfg<M, RW, PAIR>::NTHREADS, 1)
     return s;
   };
   const int CC0 = pl.CC0, NCCL = pl.CC1 - pl.CC0;
-  auto crot_of = [&](int ui) { return (int)(((unsigned)ui * 5u) % (unsigned)NCCL); };
-  auto chunk_of = [&](int ui, int cc) {  // actual channel chunk of the unit's cc-th chunk (rotated)
-    const int cr = crot_of(ui);
+  // Channel-chunk rotation (SMs do not all stream the same U image at once): a function of the
+  // strip-group PAIR and nb only, so the CTA-pair and single-CTA kernels sum every output in the
+  // same order (bitwise-identical results; the '*' path may run the single-CTA form)
+  auto chunk_of = [&](int ui, int cc) {
+    const int sgp = PAIR ? ui / pl.NB : (ui / pl.NB) >> 1, nbu = ui % pl.NB;
+    const int cr = (int)(((unsigned)(sgp * pl.NB + nbu) * 5u) % (unsigned)NCCL);
     return CC0 + (cc + cr < NCCL ? cc + cr : cc + cr - NCCL);
   };
   constexpr int PROD_WARP = NWG * 4, UPROD_WARP = PROD_WARP + 1, ISS_WARP0 = NWG * 4 + 2;

@@ -46,12 +46,13 @@ def test_host_generator_matches_oracle_generator_exactly(m, r):
 def test_plan_table():
     # paper's Table 2 Gamma_8 choices for r=4..7; r=8,9 alpha=12 (reading R7: alpha=16
     # measured 1.1e-4 max err/bound on the tcgen05 accumulator, above the 5e-5 acceptance); the
-    # paper's Gamma_4 variants for r=2 and for r=3 at C >= 256 (measured selection, reading R8)
+    # paper's Gamma_4 variant for r=2; r=3 keeps Gamma_8 at every C since the strip kernel
+    # (alpha = 8) beats the alpha = 4 base plans at C >= 256 (measured selection, reading R8)
     exp = {2: (3, 4, 0), 3: (6, 8, 0), 4: (5, 8, 0), 5: (4, 8, 0), 6: (3, 8, 0), 7: (2, 8, 0), 8: (5, 12, 0),
            9: (4, 12, 0)}
     for S, v in exp.items():
         assert i2cw.plan(S, 64) == v
-    assert i2cw.plan(3, 256) == (2, 4, 0) and i2cw.plan(3, 128) == (6, 8, 0) and i2cw.plan(2, 512) == (3, 4, 0)
+    assert i2cw.plan(3, 256) == (6, 8, 0) and i2cw.plan(3, 128) == (6, 8, 0) and i2cw.plan(2, 512) == (3, 4, 0)
     with pytest.raises(i2cw.I2CWError):
         i2cw.plan(10)
 
@@ -71,12 +72,21 @@ def test_planner_consistency(cfg):
     assert (p["P"], p["Q"]) == (P, Q)
     assert p["alpha"] == p["m"] + S - 1 and (p["m"], p["alpha"]) == i2cw.plan(S, C)[:2]
     assert p["T_r"] == -(-Q // p["m"])
-    assert p["TS"] * p["SEGS"] >= p["T_r"] and p["ROWS"] * p["PB"] >= P
-    assert p["NI"] * p["ROWS"] * p["TS"] <= 128 and 1 <= p["NI"] <= N
-    assert p["WBOX"] >= p["TS"] * p["m"] + S - 1 and p["WBOX"] <= 256 and p["HBOX"] == p["ROWS"] + R - 1
     assert p["GP"] * p["NPASS"] == p["alpha"] and p["GP"] * p["NT"] + 2 * 16 * p["GP"] <= 512
     assert p["NB"] * p["NT"] >= K and p["NCC"] * 8 >= C
     assert p["smem_bytes"] <= 227 * 1024
+    assert p["ROWS"] * p["PB"] >= P
+    if p["strip"]:
+        # strip kernel: one tile column of ROWS output rows + R-1 halo rows per 32-lane strip,
+        # 4 strips per unit (pairs of units on CTA pairs)
+        assert p["alpha"] == 8 and p["NT"] == 64 and p["ROWS"] + R - 1 <= 32 and p["HBOX"] == 32
+        assert p["NSTRIP"] == N * p["PB"] * p["T_r"] and p["tile_blocks"] == -(-p["NSTRIP"] // 4)
+        units = (-(-p["tile_blocks"] // 2) if p["pair"] else p["tile_blocks"]) * p["NB"]
+        assert p["NFULL"] <= units and p["NITEMS"] - p["NFULL"] == 2 * (units - p["NFULL"])
+        return
+    assert p["TS"] * p["SEGS"] >= p["T_r"]
+    assert p["NI"] * p["ROWS"] * p["TS"] <= 128 and 1 <= p["NI"] <= N
+    assert p["WBOX"] >= p["TS"] * p["m"] + S - 1 and p["WBOX"] <= 256 and p["HBOX"] == p["ROWS"] + R - 1
     assert p["tile_blocks"] == -(-N // p["NI"]) * p["PB"] * p["SEGS"]
     # work items (persistent schedule): whole units, then a split tail of T units as 2T
     # one-pass items, only with 2 passes, no CTA pairs and 2T <= #CTAs (148 without a GPU)
