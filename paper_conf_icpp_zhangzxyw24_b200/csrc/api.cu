@@ -195,7 +195,7 @@ void plan_strip(Plan* plp, int nsm, bool nopair) {
   constexpr int kStage = 4 * 9 * 32 * 32;           // 4 strip boxes (alpha = 8)
   const int osb = 4 * 2048, ostride = osb;  // 4 strips x 32 rows x 16 channels per output buffer
   // (U k-step slots, input stages, output buffers >= 2)
-  static int kSD[][3] = {{8, 2, 2}, {6, 2, 2}, {5, 2, 2}, {4, 2, 2}, {3, 2, 2}, {2, 2, 2}};
+  static int kSD[][3] = {{6, 2, 3}, {5, 2, 3}, {5, 2, 2}, {4, 2, 2}, {3, 2, 2}, {2, 2, 2}};
   static const bool sd_env = [] {  // I2CW_STRIP_DEPTHS=u,i,o (experiments): try these first
     const char* e = getenv("I2CW_STRIP_DEPTHS");
     int a, b, c;

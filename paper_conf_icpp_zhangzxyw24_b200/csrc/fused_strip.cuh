@@ -26,6 +26,21 @@
 
 namespace i2cw {
 
+// Light profiling (make EXTRA=-DI2CW_LTRACE=1, tools only): per-CTA cycle sums of the pipeline
+// phases kept in registers and written once at the end (pl.trace[blockIdx * 32 + k]).
+#ifndef I2CW_LTRACE
+#define I2CW_LTRACE 0
+#endif
+__device__ __forceinline__ long long lclock() {
+#if I2CW_LTRACE
+  long long t;
+  asm volatile("mov.u64 %0, %%clock64;" : "=l"(t));
+  return t;
+#else
+  return 0;
+#endif
+}
+
 template <bool PAIR>
 __device__ __forceinline__ void tmem_shift_up_warp(uint32_t taddr) {
   // PTX ".down" moves each row's 32-byte element to the row below in the matrix view, i.e. lane l
@@ -46,6 +61,9 @@ __device__ __forceinline__ void tmem_shift_up_warp(uint32_t taddr) {
 }
 
 constexpr int kStripLanes = 32;  // input rows per strip box (one TMEM subpartition)
+#ifndef I2CW_STRIP_WARPSTORE
+#define I2CW_STRIP_WARPSTORE 1  // per-warp y stores (measured +1..3% over the warpgroup-run stores, 0)
+#endif
 struct alignas(64) YMaps { CUtensorMap m[4]; };  // y store maps for runs of 1..4 strips
 
 template <int M, int RW, bool PAIR>
@@ -192,12 +210,16 @@ __global__ void __launch_bounds__(StripCfg<M, RW, PAIR>::NTHREADS, 1)
     const bool out_row = jr < pl.ROWS;  // output row of the strip (else: halo input row only)
     uint8_t* ostage = o_smem + (size_t)g * pl.NOB * pl.OSTRIDE;
     const uint32_t st_full_lead = PAIR ? mapa_shared(st_full, 0) : 0u, d_empty_lead = PAIR ? mapa_shared(d_empty, 0) : 0u;
+    long long lt[8] = {0, 0, 0, 0, 0, 0, 0, 0};  // I2CW_LTRACE sums: in_full, math, st_empty, sttm, n, d_full, epi, n
     // ---- one chunk of V (this warpgroup's chunk gc of a pass with point group PASS) ----
     auto do_chunk = [&](auto PASS_, int gc) {
       constexpr int PASS = PASS_;
       const int ist = gc % NIS;
       trace_rec(pl.trace, 0 + g, gc / NWG, l == 0);
+      long long lt0 = lclock();
       mbar_wait(&in_full[g], (gc / NWG) & 1);
+      long long lt1 = lclock();
+      lt[0] += lt1 - lt0;
       trace_rec(pl.trace, 4 + g, gc / NWG, l == 0);
       const uint8_t* box = in_smem + ((size_t)ist * 4 + sub) * SBOX;
       float2 V[GP][4];  // point tl, channel pair cp
@@ -245,8 +267,12 @@ __global__ void __launch_bounds__(StripCfg<M, RW, PAIR>::NTHREADS, 1)
         }
       }
       trace_rec(pl.trace, 8 + g, gc / NWG, l == 0);
+      lt0 = lclock();
+      lt[1] += lt0 - lt1;
       const int use = gc / NSLOT;
       if (use > 0) mbar_wait_tc<PAIR>(&st_empty[g], (use - 1) & 1);
+      lt1 = lclock();
+      lt[2] += lt1 - lt0;
       trace_rec(pl.trace, 12 + g, gc / NWG, l == 0);
       tc_fence_after();
 #pragma unroll
@@ -269,6 +295,8 @@ __global__ void __launch_bounds__(StripCfg<M, RW, PAIR>::NTHREADS, 1)
         else mbar_arrive(&st_full[g]);
       }
       trace_rec(pl.trace, 16 + g, gc / NWG, l == 0);
+      lt[3] += lclock() - lt1;
+      lt[4] += 1;
     };
 
     // ---- epilogue of one pass: y (+)= A^T M via shared memory + TMA ----
@@ -311,7 +339,10 @@ __global__ void __launch_bounds__(StripCfg<M, RW, PAIR>::NTHREADS, 1)
         }
       }
       trace_rec(pl.trace, 20 + g, 2 * E.gpass, l == 0);
+      const long long le0 = lclock();
       mbar_wait_tc<PAIR>(d_full, E.gpass & 1);
+      const long long le1 = lclock();
+      lt[5] += le1 - le0;
       trace_rec(pl.trace, 20 + g, 2 * E.gpass + 1, l == 0);
       tc_fence_after();
       const int cbase = g * CPW;
@@ -339,6 +370,74 @@ __global__ void __launch_bounds__(StripCfg<M, RW, PAIR>::NTHREADS, 1)
           }
         }
       });
+#if I2CW_STRIP_WARPSTORE
+      // Per-warp stores: warp (g, sub) stages its own strip's rows (64-byte rows, 64B swizzle,
+      // conflict-free) and its lane 0 issues that strip's box (16 channels x 1 tile x ROWS rows)
+      // per output column -- no warpgroup barrier, each warp tracks its own bulk groups.
+      {
+        const bool mine = sub < nvalid;
+        Strip ms = strip_at(E.sg0 + (mine ? sub : 0));
+        const uint32_t wbase = (uint32_t)(sub * Cfg::TSTRIDE + jr * 64);
+        const uint32_t wxor = ((wbase >> 7) & 3u) << 4;
+        if (lane32 == 0) {
+          bulk_wait_group_read_dyn(pl.NOB - 1);
+          if (PASS > 0 && !E.split) bulk_wait_group_all();  // this warp's pass-0 stores of the unit landed
+        }
+        __syncwarp();
+        const bool store = PASS == 0 && !E.split && !pl.ACCUM;
+        static_for<M>([&](auto I_) {
+          constexpr int i = I_;
+          const int ob = i % pl.NOB;
+          uint8_t* stg = ostage + (size_t)ob * pl.OSTRIDE;
+#pragma unroll
+          for (int j = 0; j < CPW / 4; ++j) {
+            float2 o[2] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
+            static_for<GP / 2>([&](auto Q_) {
+              constexpr int idx0 = PASS * GP + 2 * (int)Q_;
+              constexpr int tl0 = 2 * (int)Q_;
+              if constexpr (idx0 == 0) {
+                constexpr float c0 = T::AT(i, 0), c1 = T::AT(i, A - 1);
+#pragma unroll
+                for (int e = 0; e < 2; ++e) {
+                  const float2 m0 = make_float2(mv[tl0][4 * j + 2 * e], mv[tl0][4 * j + 2 * e + 1]);
+                  const float2 m1 = make_float2(mv[tl0 + 1][4 * j + 2 * e], mv[tl0 + 1][4 * j + 2 * e + 1]);
+                  if constexpr (c0 != 0.f) o[e] = __ffma2_rn(make_float2(c0, c0), m0, o[e]);
+                  if constexpr (c1 != 0.f) o[e] = __ffma2_rn(make_float2(c1, c1), m1, o[e]);
+                }
+              } else {
+                constexpr float ca = T::AT(i, point_of(idx0, A));
+                constexpr int src = (i % 2 == 0) ? tl0 : tl0 + 1;
+#pragma unroll
+                for (int e = 0; e < 2; ++e) {
+                  const float2 mz = make_float2(mv[src][4 * j + 2 * e], mv[src][4 * j + 2 * e + 1]);
+                  if constexpr (ca == 1.f) o[e] = __fadd2_rn(o[e], mz);
+                  else if constexpr (ca != 0.f) o[e] = __ffma2_rn(make_float2(ca, ca), mz, o[e]);
+                }
+              }
+            });
+            if (out_row && mine)
+              *reinterpret_cast<float4*>(stg + ((wbase + (uint32_t)j * 16u) ^ wxor)) = make_float4(o[0].x, o[0].y, o[1].x, o[1].y);
+          }
+          fence_proxy_async_smem();
+          __syncwarp();
+          if (lane32 == 0) {
+            if (mine && !ABL(32)) {
+              const uint8_t* src = stg + sub * Cfg::TSTRIDE;
+              if (store) tma_store_4d(&ym.m[0], src, E.nb * NT + cbase, ms.tw * M + i, ms.rb * pl.ROWS, ms.n);
+              else tma_reduce_add_4d(&ym.m[0], src, E.nb * NT + cbase, ms.tw * M + i, ms.rb * pl.ROWS, ms.n);
+            }
+            bulk_commit_group();
+            // the buffer the next column writes was last read by column i + 1 - NOB
+            bulk_wait_group_read_dyn(pl.NOB - 1);
+          }
+          __syncwarp();
+        });
+        if (lane32 == 0) bulk_wait_group_read<0>();
+        lt[6] += lclock() - le1;
+        lt[7] += 1;
+        return;
+      }
+#endif
       trace_rec(pl.trace, 28 + (g == 0 ? 3 : 0), 0, false);
       if (l == 0) {
         bulk_wait_group_read_dyn(pl.NOB - 1);
@@ -401,6 +500,8 @@ __global__ void __launch_bounds__(StripCfg<M, RW, PAIR>::NTHREADS, 1)
         trace_rec(pl.trace, 24 + g, E.gpass * 8 + i, l == 0);
       });
       if (l == 0) bulk_wait_group_read<0>();
+      lt[6] += lclock() - le1;
+      lt[7] += 1;
       trace_rec(pl.trace, 24 + g, E.gpass * 8 + 7, l == 0);
     };
     auto epilogue = [&](const Epi& E) {
@@ -432,6 +533,10 @@ __global__ void __launch_bounds__(StripCfg<M, RW, PAIR>::NTHREADS, 1)
       }
     }
     if (pend) epilogue(pe);
+#if I2CW_LTRACE
+    if (pl.trace != nullptr && lane32 == 0 && sub == 0)
+      for (int k = 0; k < 8; ++k) pl.trace[(size_t)blockIdx.x * 48 + g * 8 + k] = lt[k];
+#endif
   } else {
     setmaxnreg_dec<56>();
     if (warp == PROD_WARP) {
@@ -453,6 +558,7 @@ __global__ void __launch_bounds__(StripCfg<M, RW, PAIR>::NTHREADS, 1)
               trace_rec(pl.trace, 31, gcp);
               const int ca = chunk_of(I.ui, cc);
               uint64_t* full = &in_full[gcp & 3];
+              if (ABL(8)) { mbar_arrive(full); if (++ist == NIS) { ist = 0; iph ^= 1; first = 0; } continue; }
               mbar_expect_tx(full, 4u * SBOX);
 #pragma unroll
               for (int s = 0; s < 4; ++s)
@@ -488,6 +594,7 @@ __global__ void __launch_bounds__(StripCfg<M, RW, PAIR>::NTHREADS, 1)
               const int ca = chunk_of(I.ui, cc);
               for (int fh = 0; fh < R; ++fh) {
                 if (!first) mbar_wait_tc<PAIR>(&u_empty[us], uph ^ 1);
+                if (ABL(16)) { mbar_arrive(&u_full[us]); if (++us == NUS) { us = 0; uph ^= 1; first = 0; } continue; }
                 mbar_expect_tx(&u_full[us], UBYTES);
                 bulk_load(u_smem + (size_t)us * UBYTES, src0 + (size_t)(ca * R + fh) * kstride, UBYTES, &u_full[us]);
                 if (++us == NUS) { us = 0; uph ^= 1; first = 0; }
@@ -503,6 +610,8 @@ __global__ void __launch_bounds__(StripCfg<M, RW, PAIR>::NTHREADS, 1)
       constexpr uint32_t idesc = idesc_tf32(PAIR ? 256 : 128, NT);
       const uint64_t bdesc0 = umma_desc_kmajor_noswizzle(smem_u32(u_smem), BROWS * 16, 128);
       int us = 0, uph = 0, gc = 0, gpass = 0;
+      long long ilt[4] = {0, 0, 0, 0};  // I2CW_LTRACE: st_full waits, u_full waits, d_empty waits, total
+      const long long ilt_start = lclock();
       if (PAIR && rank == 1) {
         // pair peer: forward "my U half landed" to the leader's U slot (off the critical path:
         // the U ring runs ahead)
@@ -512,7 +621,7 @@ __global__ void __launch_bounds__(StripCfg<M, RW, PAIR>::NTHREADS, 1)
             const Item I = item_at(it);
             for (int pass = I.pb; pass < I.pe; ++pass)
               for (int k = 0; k < NCCL * R; ++k) {
-                mbar_wait_tc<PAIR>(&u_full[us], uph);
+                mbar_wait(&u_full[us], uph);  // this CTA's own U half (local TMA completion)
                 mbar_arrive_remote(lead_ufull + 8u * (uint32_t)us);
                 if (++us == NUS) { us = 0; uph ^= 1; }
               }
@@ -523,18 +632,24 @@ __global__ void __launch_bounds__(StripCfg<M, RW, PAIR>::NTHREADS, 1)
         const Item I = item_at(it);
         for (int pass = I.pb; pass < I.pe; ++pass, ++gpass) {
           if (gpass > 0) {
+            const long long dt0 = lclock();
             mbar_wait_tc<PAIR>(d_empty, (gpass - 1) & 1);
+            ilt[2] += lclock() - dt0;
             tc_fence_after();
           }
           for (int cc = 0; cc < NCCL; ++cc, ++gc) {
             const int slot = gc & (NSLOT - 1);
             trace_rec(pl.trace, 28, gc, iss == 0 && lane32 == 0);
+            long long it0 = lclock();
             mbar_wait_tc<PAIR>(&st_full[slot], (gc / NSLOT) & 1);
+            ilt[0] += lclock() - it0;
             trace_rec(pl.trace, 29, gc, iss == 0 && lane32 == 0);
             tc_fence_after();
             const uint32_t va = tbase + VCOL + (uint32_t)slot * GP * 16;
             for (int fh = 0; fh < R; ++fh) {
-              mbar_wait(&u_full[us], uph);
+              it0 = lclock();
+              mbar_wait_tc<PAIR>(&u_full[us], uph);  // pair: both halves (the peer's arrives remotely)
+              ilt[1] += lclock() - it0;
               tc_fence_after();
               const uint64_t bk = bdesc0 + (uint64_t)((us * UBYTES) >> 4);
               if (!ABL(2)) {
@@ -571,6 +686,11 @@ __global__ void __launch_bounds__(StripCfg<M, RW, PAIR>::NTHREADS, 1)
           else mma_commit_warp(d_full);
         }
       }
+#if I2CW_LTRACE
+      ilt[3] = lclock() - ilt_start;
+      if (pl.trace != nullptr && lane32 == 0 && iss == 0)
+        for (int k = 0; k < 4; ++k) pl.trace[(size_t)blockIdx.x * 48 + 32 + k] = ilt[k];
+#endif
       __syncwarp();
     }
   }
