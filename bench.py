@@ -418,7 +418,9 @@ def main():
             "config": {"workload": desc, "name": args.config, "global_batch": N_job,
                        "per_gpu_batch": N if args.scaling == "weak" else f"{N_cfg // world}-{-(-N_cfg // world)}",
                        "parallelism": f"batch-sharded x{world} (shard_range), no collective in the timed region",
-                       "F(m,r)": f"F({p['m']},{S}) alpha={p['alpha']}", "l2": "flushed (256 MiB memset) before every step",
+                       "F(m,r)": f"F({p['m']},{S}) alpha={p['alpha']}",
+                       "kernel": ("fused_strip_kernel (CTA pairs)" if p.get("pair") else "fused_strip_kernel") if p.get("strip")
+                       else "fused_tc_kernel", "l2": "flushed (256 MiB memset) before every step",
                        "inputs": "x[n] ~ U[-1,1) seeded 1000+n per global image n (on device), w ~ U[-1,1) seed 7",
                        "step": f"i2cw_{'de' if is_deconv else ''}conv2d_nhwc (C ABI one-shot call: filter transform + fused kernel)"},
             "roofline": rf,
@@ -471,7 +473,8 @@ def roofline(i2cw, cfg, N, p, t_launch, pk, pk_src):
     achieved = f_tc / t_launch / 1e12
     hbm_bytes = 4 * (N * H * W * C + N * P * Q * K) + (i2cw.filter_bytes(K, C, R, S) - 256)
     rf = {"bound": "tensor", "achieved": achieved, "peak": tf32_peak, "unit": "TFLOP/s",
-          "frac": achieved / tf32_peak, "kernel": "fused_tc_kernel", "kernel_ms": t_launch * 1e3,
+          "frac": achieved / tf32_peak, "kernel": "fused_strip_kernel" if p.get("strip") else "fused_tc_kernel",
+          "kernel_ms": t_launch * 1e3,
           "work": "3xTF32 UMMA flops 6*alpha*N*P*(Q/m)*K*R*C per launch",
           "peak_src": f"{pk_src}: bf16_tflops {pk['bf16_tflops']} x 0.5 (tf32/bf16 nominal)",
           "hbm_frac": hbm_bytes / t_launch / 1e9 / pk["hbm_gbs"],

@@ -3,7 +3,7 @@
 # of the cfg2 bench step. Usage (under gpurun): bash tools/ncu_all.sh TAG
 TAG=${1:-r02}; OUT=gpurun_out; mkdir -p $OUT
 for c in ${CFGS:-cfg2 cfg3-r2 cfg3-r3 cfg3-r4 cfg3-r5 cfg3-r6 cfg3-r7 cfg3-r8 cfg3-r9 cfg4-r5 cfg4-r7 cfg5a cfg5b-c64 cfg5b-c128 cfg5b-c256 cfg5b-c512}; do
-  timeout 600 ncu --set full --clock-control none --import-source on -k regex:fused_tc -s 2 -c 1 -f \
+  timeout 600 ncu --set full --clock-control none --import-source on -k regex:"fused_tc|fused_strip" -s 2 -c 1 -f \
       -o $OUT/ncu_${TAG}_$c python tools/ncu_one.py $c > $OUT/ncu_${TAG}_$c.log 2>&1
   echo "$c rc=$?"
   # summaries travel back; the reports do not (the returned gpurun_out/ is capped at 64 MiB),
