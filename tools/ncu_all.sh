@@ -11,6 +11,6 @@ for c in ${CFGS:-cfg2 cfg3-r2 cfg3-r3 cfg3-r4 cfg3-r5 cfg3-r6 cfg3-r7 cfg3-r8 cf
   python tools/ncu_summary.py $OUT/ncu_${TAG}_$c.ncu-rep $c $OUT/traffic_${TAG}.json > $OUT/ncu_${TAG}_${c}_summary.md 2>&1
   [ "$c" = "${KEEP:-cfg2}" ] || rm -f $OUT/ncu_${TAG}_$c.ncu-rep
 done
-timeout 300 ncu --metrics gpu__time_duration.sum --clock-control none -c 80 --csv --log-file $OUT/launches_${TAG}_cfg2.csv \
+timeout 300 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"fused|filter|zero|ksum" -c 24 --csv --log-file $OUT/launches_${TAG}_cfg2.csv \
     python bench.py --steps 5 --warmup 3 --no-cpu --no-e2e --no-sweep --no-peak > /dev/null 2>&1
 echo "launch list rc=$?"
