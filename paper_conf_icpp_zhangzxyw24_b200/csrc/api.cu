@@ -194,22 +194,37 @@ void plan_strip(Plan* plp, int nsm, bool nopair) {
   const int kUB = 4 * 2 * (spair ? 32 : 64) * 32;  // this CTA's U k-step (alpha = 8, GP = 4)
   constexpr int kStage = 4 * 9 * 32 * 32;           // 4 strip boxes (alpha = 8)
   const int osb = 4 * 2048, ostride = osb;  // 4 strips x 32 rows x 16 channels per output buffer
-  // (U k-step slots, input stages, output buffers >= 2)
+  // U ring: one k-step per slot. One slot per chunk (KU = R: one barrier wait and commit per
+  // chunk instead of R) fits only 2 slots and measured 4-5% slower on cfg2 / c128 (the U stream's
+  // latency shows through one chunk of lookahead); I2CW_STRIP_KU=2 selects it (experiments).
+  // Candidates: (U slots, input stages, output buffers >= 2).
   static int kSD[][3] = {{6, 2, 3}, {5, 2, 3}, {5, 2, 2}, {4, 2, 2}, {3, 2, 2}, {2, 2, 2}};
+  static int kSDc[][3] = {{3, 2, 3}, {2, 2, 3}, {3, 2, 2}, {2, 2, 2}};
   static const bool sd_env = [] {  // I2CW_STRIP_DEPTHS=u,i,o (experiments): try these first
     const char* e = getenv("I2CW_STRIP_DEPTHS");
     int a, b, c;
-    if (e && sscanf(e, "%d,%d,%d", &a, &b, &c) == 3 && b >= 1 && c >= 2) { kSD[0][0] = a; kSD[0][1] = b; kSD[0][2] = c; }
+    if (e && sscanf(e, "%d,%d,%d", &a, &b, &c) == 3 && b >= 1 && c >= 2) {
+      kSD[0][0] = a; kSD[0][1] = b; kSD[0][2] = c;
+      kSDc[0][0] = a; kSDc[0][1] = b; kSDc[0][2] = c;
+    }
     return e != nullptr;
   }();
   (void)sd_env;
-  int sel = -1, smem = 0;
-  for (int d = 0; d < (int)(sizeof(kSD) / sizeof(kSD[0])); ++d) {
-    const int bar_bytes = 8 * (4 + kSD[d][1] + 10 + 2 * kSD[d][0]) + 32 + 4 * 4 * 16;  // + slot, epilogue op table
-    smem = kSD[d][0] * kUB + kSD[d][1] * kStage + 4 * kSD[d][2] * ostride + bar_bytes;
-    if (smem <= kSmemBudget) { sel = d; break; }
+  static const int ku_env = [] { const char* e = getenv("I2CW_STRIP_KU"); return e ? atoi(e) : 0; }();
+  int sel = -1, smem = 0, ku = 1;
+  for (int pass = 0; pass < 2 && sel < 0; ++pass) {
+    ku = pass == 0 ? pl.R : 1;
+    if (pass == 0 && (ku_env < 2 || pl.R == 1)) continue;
+    const int(*cand)[3] = pass == 0 ? kSDc : kSD;
+    const int ncand = pass == 0 ? 4 : 6;
+    for (int d = 0; d < ncand; ++d) {
+      const int bar_bytes = 8 * (4 + cand[d][1] + 10 + 2 * cand[d][0]) + 32 + 4 * 4 * 16;  // + slot, op table
+      smem = cand[d][0] * ku * kUB + cand[d][1] * kStage + 4 * cand[d][2] * ostride + bar_bytes;
+      if (smem <= kSmemBudget) { sel = d; break; }
+    }
   }
   if (sel < 0) return;
+  const int(*kSel)[3] = ku > 1 ? kSDc : kSD;
   pl.strip = 1;
   pl.pair = spair;
   pl.NSTRIP = (int)nstrip;
@@ -221,9 +236,10 @@ void plan_strip(Plan* plp, int nsm, bool nopair) {
   pl.HBOX = kStripLanes;
   pl.WBOX = pl.alpha;
   pl.tile_blocks = sgroups;
-  pl.NUS = kSD[sel][0];
-  pl.NIS = kSD[sel][1];
-  pl.NOB = kSD[sel][2];
+  pl.KU = ku;
+  pl.NUS = kSel[sel][0];
+  pl.NIS = kSel[sel][1];
+  pl.NOB = kSel[sel][2];
   pl.OSB = osb;
   pl.OSTRIDE = ostride;
   pl.BOXB = kStage;

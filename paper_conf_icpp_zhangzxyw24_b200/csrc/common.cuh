@@ -57,6 +57,7 @@ struct Plan {
   int strip;            // 1: strip kernel (fused_strip.cuh): one input-row transform per chunk, TMEM row
                         // shifts between filter rows; ROWS = valid rows per strip, TS = 4 strips per unit
   int NSTRIP;           // strip kernel: strips = N * PB * T_r (tile column tw fastest)
+  int KU;               // strip kernel: k-steps per U ring slot (R: one barrier round trip per chunk, or 1)
   int ablate;           // DEBUG timing ablation (I2CW_ABLATE, results wrong): 1 no transform math,
                         // 2 no MMAs, 4 no epilogue math/stores; 0 in production
   unsigned long long* trace;  // debug timeline of CTA 0 (nullptr = off), see i2cw_debug_trace

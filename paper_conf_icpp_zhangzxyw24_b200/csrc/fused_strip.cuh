@@ -104,7 +104,7 @@ struct StripCfg {
 // stream from L2 and the B-operand reads from shared memory). The leader (rank 0) issues all
 // MMAs and shifts; the peer's warps arrive remotely on the leader's V / accumulator barriers and
 // a peer thread forwards "my U half landed"; commits are multicast to both CTAs.
-template <int M, int RW, bool PAIR>
+template <int M, int RW, bool PAIR, bool UCH>
 __global__ void __launch_bounds__(StripCfg<M, RW, PAIR>::NTHREADS, 1)
     fused_strip_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__ YMaps ym,
                        const __grid_constant__ Plan pl, const float* __restrict__ u) {
@@ -116,11 +116,13 @@ __global__ void __launch_bounds__(StripCfg<M, RW, PAIR>::NTHREADS, 1)
   constexpr int NISS = Cfg::NISS, PPI = Cfg::PPI, VCOL = Cfg::VCOL, NT = Cfg::NT;
   constexpr uint32_t UBYTES = Cfg::UBYTES, SBOX = Cfg::SBOX;
   constexpr int CPW = NT / NWG;  // epilogue channels per warpgroup (64-byte staging rows)
-  const int NIS = pl.NIS, NUS = pl.NUS, R = pl.R;
+  const int NIS = pl.NIS, NUS = pl.NUS, R = pl.R, KU = pl.KU;
+  constexpr bool uchunk = UCH;                    // one U slot per chunk (KU = R k-steps), else per k-step
+  const uint32_t USLOT = (uint32_t)KU * UBYTES;  // one U ring slot: KU k-steps
 
   extern __shared__ __align__(1024) uint8_t smem[];
-  uint8_t* u_smem = smem;                                        // [NUS][UBYTES]
-  uint8_t* o_smem = u_smem + (size_t)NUS * UBYTES;               // [NWG][NOB][OSTRIDE]
+  uint8_t* u_smem = smem;                                        // [NUS][KU][UBYTES]
+  uint8_t* o_smem = u_smem + (size_t)NUS * USLOT;                // [NWG][NOB][OSTRIDE]
   uint8_t* in_smem = o_smem + (size_t)NWG * pl.NOB * pl.OSTRIDE;  // [NIS][4][SBOX]
   uint64_t* bars = reinterpret_cast<uint64_t*>(in_smem + (size_t)NIS * 4 * SBOX);
   // Input ring: the data stages rotate with gc mod NIS, but "chunk gc landed" is signalled on
@@ -222,17 +224,36 @@ __global__ void __launch_bounds__(StripCfg<M, RW, PAIR>::NTHREADS, 1)
       lt[0] += lt1 - lt0;
       trace_rec(pl.trace, 4 + g, gc / NWG, l == 0);
       const uint8_t* box = in_smem + ((size_t)ist * 4 + sub) * SBOX;
-      float2 V[GP][4];  // point tl, channel pair cp
+      // All 16 loads first, then release the box, then the B^T math from registers: the stage is
+      // held only for the loads, so the producer refills it while the math runs. The release
+      // waits on a branch that reads a sum of every loaded vector (an arrive issued right after the
+      // LDS instructions can overtake them -- ptxas adds no wait -- and the next TMA fill would
+      // land under the reads); the bit pattern is a signalling NaN, which no sum produces.
+      float2 d2[2][A][2];
 #pragma unroll
-      for (int h = 0; h < 2; ++h) {
-        float2 d[A][2];
+      for (int h = 0; h < 2; ++h)
 #pragma unroll
         for (int j = 0; j < A; ++j) {
           const uint32_t o = rofs + (uint32_t)j * 32;  // 32B swizzle: bit 4 ^= bit 7
           const float4 v = *reinterpret_cast<const float4*>(box + ((o ^ ((o >> 3) & 16u)) ^ (uint32_t)(h << 4)));
-          d[j][0] = make_float2(v.x, v.y);
-          d[j][1] = make_float2(v.z, v.w);
+          d2[h][j][0] = make_float2(v.x, v.y);
+          d2[h][j][1] = make_float2(v.z, v.w);
         }
+      {
+        float2 acc2 = make_float2(0.f, 0.f);
+#pragma unroll
+        for (int h = 0; h < 2; ++h)
+#pragma unroll
+          for (int j = 0; j < A; ++j) acc2 = __fadd2_rn(acc2, __fadd2_rn(d2[h][j][0], d2[h][j][1]));
+        if (__float_as_uint(acc2.x + acc2.y) != 0x7f800001u) {
+          __syncwarp();
+          if (lane32 == 0) mbar_arrive(&in_empty[ist]);
+        }
+      }
+      float2 V[GP][4];  // point tl, channel pair cp
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const float2 (&d)[A][2] = d2[h];
         static_for<GP / 2>([&](auto Q_) {
           constexpr int idx0 = PASS * GP + 2 * (int)Q_;
           constexpr int tl0 = 2 * (int)Q_;
@@ -250,21 +271,6 @@ __global__ void __launch_bounds__(StripCfg<M, RW, PAIR>::NTHREADS, 1)
             }
           }
         });
-      }
-      // Release the box once every load of this lane has completed: the branch reads a sum of
-      // all 16 loaded vectors (an arrive issued right after the LDS instructions can overtake
-      // them -- ptxas adds no wait -- and the next TMA fill would land under the reads). The
-      // bit pattern is a signalling NaN, which no sum produces, so the branch is always taken.
-      {
-        float2 acc2 = make_float2(0.f, 0.f);
-#pragma unroll
-        for (int t = 0; t < GP; ++t)
-#pragma unroll
-          for (int cp = 0; cp < 4; ++cp) acc2 = __fadd2_rn(acc2, V[t][cp]);
-        if (__float_as_uint(acc2.x + acc2.y) != 0x7f800001u) {
-          __syncwarp();
-          if (lane32 == 0) mbar_arrive(&in_empty[ist]);
-        }
       }
       trace_rec(pl.trace, 8 + g, gc / NWG, l == 0);
       lt0 = lclock();
@@ -593,11 +599,16 @@ __global__ void __launch_bounds__(StripCfg<M, RW, PAIR>::NTHREADS, 1)
             for (int cc = 0; cc < NCCL; ++cc) {
               const int ca = chunk_of(I.ui, cc);
               for (int fh = 0; fh < R; ++fh) {
-                if (!first) mbar_wait_tc<PAIR>(&u_empty[us], uph ^ 1);
-                if (ABL(16)) { mbar_arrive(&u_full[us]); if (++us == NUS) { us = 0; uph ^= 1; first = 0; } continue; }
-                mbar_expect_tx(&u_full[us], UBYTES);
-                bulk_load(u_smem + (size_t)us * UBYTES, src0 + (size_t)(ca * R + fh) * kstride, UBYTES, &u_full[us]);
-                if (++us == NUS) { us = 0; uph ^= 1; first = 0; }
+                const int kin = uchunk ? fh : 0;  // position in the U slot
+                if (kin == 0) {
+                  if (!first) mbar_wait_tc<PAIR>(&u_empty[us], uph ^ 1);
+                  if (ABL(16)) mbar_arrive(&u_full[us]);
+                  else mbar_expect_tx(&u_full[us], USLOT);
+                }
+                if (!ABL(16))
+                  bulk_load(u_smem + (size_t)us * USLOT + (size_t)kin * UBYTES, src0 + (size_t)(ca * R + fh) * kstride,
+                            UBYTES, &u_full[us]);
+                if (!uchunk || fh == R - 1) { if (++us == NUS) { us = 0; uph ^= 1; first = 0; } }
               }
             }
           }
@@ -620,7 +631,7 @@ __global__ void __launch_bounds__(StripCfg<M, RW, PAIR>::NTHREADS, 1)
           for (int it = unit0; it < NITEMS; it += ustride) {
             const Item I = item_at(it);
             for (int pass = I.pb; pass < I.pe; ++pass)
-              for (int k = 0; k < NCCL * R; ++k) {
+              for (int k = 0; k < NCCL * (uchunk ? 1 : R); ++k) {
                 mbar_wait(&u_full[us], uph);  // this CTA's own U half (local TMA completion)
                 mbar_arrive_remote(lead_ufull + 8u * (uint32_t)us);
                 if (++us == NUS) { us = 0; uph ^= 1; }
@@ -647,11 +658,14 @@ __global__ void __launch_bounds__(StripCfg<M, RW, PAIR>::NTHREADS, 1)
             tc_fence_after();
             const uint32_t va = tbase + VCOL + (uint32_t)slot * GP * 16;
             for (int fh = 0; fh < R; ++fh) {
-              it0 = lclock();
-              mbar_wait_tc<PAIR>(&u_full[us], uph);  // pair: both halves (the peer's arrives remotely)
-              ilt[1] += lclock() - it0;
-              tc_fence_after();
-              const uint64_t bk = bdesc0 + (uint64_t)((us * UBYTES) >> 4);
+              const int kin = uchunk ? fh : 0;
+              if (kin == 0) {
+                it0 = lclock();
+                mbar_wait_tc<PAIR>(&u_full[us], uph);  // pair: both halves (the peer's arrives remotely)
+                ilt[1] += lclock() - it0;
+                tc_fence_after();
+              }
+              const uint64_t bk = bdesc0 + (uint64_t)((us * USLOT + kin * UBYTES) >> 4);
               if (!ABL(2)) {
 #pragma unroll
               for (int prod = 0; prod < 3; ++prod) {
@@ -666,9 +680,11 @@ __global__ void __launch_bounds__(StripCfg<M, RW, PAIR>::NTHREADS, 1)
                 }
               }
               }
-              if constexpr (PAIR) mma_commit2_warp(&u_empty[us]);
-              else mma_commit_warp(&u_empty[us]);
-              if (++us == NUS) { us = 0; uph ^= 1; }
+              if (!uchunk || fh == R - 1) {
+                if constexpr (PAIR) mma_commit2_warp(&u_empty[us]);
+                else mma_commit_warp(&u_empty[us]);
+                if (++us == NUS) { us = 0; uph ^= 1; }
+              }
               if (fh + 1 < R && !ABL(2)) {  // next filter row: lane j takes lane j+1's input row
 #pragma unroll
                 for (int pi = 0; pi < PPI; ++pi) {
@@ -709,10 +725,10 @@ __global__ void __launch_bounds__(StripCfg<M, RW, PAIR>::NTHREADS, 1)
 }
 
 template <int M, int RW, bool PAIR>
-static cudaError_t launch_strip_t(const CUtensorMap& xmap, const YMaps& ym, const Plan& pl, const float* u,
+static cudaError_t launch_strip_t2(const CUtensorMap& xmap, const YMaps& ym, const Plan& pl, const float* u,
                                   cudaStream_t stream) {
   using Cfg = StripCfg<M, RW, PAIR>;
-  auto kern = fused_strip_kernel<M, RW, PAIR>;
+  auto kern = pl.KU > 1 ? fused_strip_kernel<M, RW, PAIR, true> : fused_strip_kernel<M, RW, PAIR, false>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, pl.smem_bytes);
   if (e != cudaSuccess) return e;
   cudaLaunchConfig_t cfg = {};

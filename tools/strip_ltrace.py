@@ -29,9 +29,9 @@ for name in sys.argv[1:] or ["cfg2"]:
         print(f"  WG{g}: chunks/CTA {n.mean():.1f}; per chunk: in_full {np.mean(b[:,0]/n):.0f} math {np.mean(b[:,1]/n):.0f} "
               f"st_empty {np.mean(b[:,2]/n):.0f} sttm {np.mean(b[:,3]/n):.0f}; per pass: d_full {np.mean(b[:,5]/ne):.0f} epi {np.mean(b[:,6]/ne):.0f}; "
               f"total WG busy {np.mean(b[:,0]+b[:,1]+b[:,2]+b[:,3]+b[:,5]+b[:,6]):.0f}")
-    iss = T[:, 32:36].astype(float)
-    lead = iss[:, 3] > 0
-    iss = iss[lead]
-    nch = T[lead, 4] * 4
-    print(f"  issuer (leaders {lead.sum()}): total {iss[:,3].mean():.0f} cycles; st_full waits {iss[:,0].mean():.0f}, "
+    pair = i2cw.debug_plan(kind, N, H, W, C, K, R, S, ph, pw)["pair"]
+    Tl = T[0::2] if pair else T  # pair: the even CTA of each pair is the MMA leader
+    iss = Tl[:, 32:36].astype(float)
+    nch = Tl[:, 4] * 4
+    print(f"  issuer (leaders {len(Tl)}): total {iss[:,3].mean():.0f} cycles; st_full waits {iss[:,0].mean():.0f}, "
           f"u_full waits {iss[:,1].mean():.0f}, d_empty waits {iss[:,2].mean():.0f}; per chunk: st_full {np.mean(iss[:,0]/nch):.0f} u_full {np.mean(iss[:,1]/nch):.0f}")
