@@ -210,9 +210,12 @@ I2CW_API int i2cw_set_device(int device);
  * Host-side introspection (no GPU needed).
  * i2cw_plan: the Winograd choice for filter width S and C input channels: m outputs,
  *   alpha = m+S-1 states, and the alpha = 16 point set (0 paper, 1 alt; reading R7).
- *   S = 2: Gamma4(3,2); S = 3: Gamma4(2,3) when C >= 256, else Gamma8(6,3); S = 4..7: Gamma8;
- *   S = 8, 9: alpha = 12 (measured selection, reading R8). The 3D and 1xTF32 calls use
- *   alpha = 8 for S = 2, 3. Returns I2CW_EUNSUPPORTED for S outside [2, 9], EINVAL for C <= 0.
+ *   S = 2: Gamma4(3,2); S = 3: Gamma8(6,3) (Gamma4(2,3) for C >= 256 only when the strip kernel
+ *   is disabled with I2CW_STRIP=0); S = 4..7: Gamma8; S = 8, 9: alpha = 12 (measured selection,
+ *   DESIGN.md reading R8). The 3D and 1xTF32 calls use alpha = 8 for S = 2, 3. The planner runs
+ *   the strip kernel or the base kernel for a call; both read the same U layout
+ *   produced by i2cw_filter_transform and give results within the same bound. Returns
+ *   I2CW_EUNSUPPORTED for S outside [2, 9], EINVAL for C <= 0.
  * i2cw_transform_matrices_rational: the exact Cook-Toom matrices of F(m, r)
  *   (§5.3, Figure 5) as int64 numerator/denominator
  *   pairs, row-major: AT (m x alpha), G (alpha x r), BT (alpha x alpha), with

@@ -574,7 +574,7 @@ __global__ void __launch_bounds__(StripCfg<M, RW, PAIR>::NTHREADS, 1)
       for (int k = 0; k < 8; ++k) pl.trace[(size_t)blockIdx.x * 48 + g * 8 + k] = lt[k];
 #endif
   } else {
-    setmaxnreg_dec<56>();
+    setmaxnreg_dec<64>();
     if (warp == PROD_WARP) {
       // ====================== input strip boxes (TMA) ======================
       if (lane32 == 0) {

@@ -312,8 +312,8 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
   const uint32_t tbase = *tmem_slot;
 
   // Register split (640-thread configs launch at 96 registers per thread): the transform /
-  // epilogue warpgroups take 104, the producer + issuer warpgroup keeps 56 (the CTA's pool is
-  // only what the launch allocated: 4 x 128 x 8 <= 128 x 40 released).
+  // epilogue warpgroups take 104, the producer + issuer warpgroup keeps 64 (the CTA's pool is
+  // only what the launch allocated: 4 x 128 x 8 = 128 x 32 released).
   constexpr bool kRegSplit = Cfg::NTHREADS == 640;
   if (warp < NWG * 4) {
     if constexpr (kRegSplit) setmaxnreg_inc<104>();
@@ -649,7 +649,7 @@ __global__ void __launch_bounds__(TcCfg<M, RW, NT, PAIR>::NTHREADS, 1)
     });
     }  // units
   } else {
-   if constexpr (kRegSplit) setmaxnreg_dec<56>();
+   if constexpr (kRegSplit) setmaxnreg_dec<64>();
    if (warp == PROD_WARP) {
     // ====================== input-row TMA producer ======================
     if (lane32 == 0) {
