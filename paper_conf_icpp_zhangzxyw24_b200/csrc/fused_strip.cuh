@@ -339,10 +339,11 @@ __global__ void __launch_bounds__(StripCfg<M, RW, PAIR>::NTHREADS, 1)
     struct Epi { int gpass, pass, sg0, nb; bool split; };
     auto do_epilogue = [&](auto PASS_, const Epi& E) {
       constexpr int PASS = PASS_;
+      const int nvalid = max(0, min(4, pl.NSTRIP - E.sg0));  // 0: a pair's idle half
+#if !I2CW_STRIP_WARPSTORE
       // runs of the unit: strips with the same (n, rb) (a run starts at s = 0 or where tw = 0).
       // This warp's strip sub is tile t = sub - r0 of the run [r0, r0 + rl); the run's staging
       // region starts at r0 * TSTRIDE and holds [row][rl tiles][16 ch] (the box image of map rl)
-      const int nvalid = max(0, min(4, pl.NSTRIP - E.sg0));  // 0: a pair's idle half
       int r0 = 0, rl = 1;
       for (int s = 1; s <= sub; ++s)
         if (s < nvalid && strip_at(E.sg0 + s).tw == 0) r0 = s;
@@ -374,6 +375,7 @@ __global__ void __launch_bounds__(StripCfg<M, RW, PAIR>::NTHREADS, 1)
           ops[nops - 1].x = cur_s | ((cur_L - 1) << 8);
         }
       }
+#endif
       trace_rec(pl.trace, 20 + g, 2 * E.gpass, l == 0);
       const long long le0 = lclock();
       mbar_wait_tc<PAIR>(d_full, E.gpass & 1);
@@ -474,6 +476,7 @@ __global__ void __launch_bounds__(StripCfg<M, RW, PAIR>::NTHREADS, 1)
         return;
       }
 #endif
+#if !I2CW_STRIP_WARPSTORE
       trace_rec(pl.trace, 28 + (g == 0 ? 3 : 0), 0, false);
       if (l == 0) {
         bulk_wait_group_read_dyn(pl.NOB - 1);
@@ -539,6 +542,7 @@ __global__ void __launch_bounds__(StripCfg<M, RW, PAIR>::NTHREADS, 1)
       lt[6] += lclock() - le1;
       lt[7] += 1;
       trace_rec(pl.trace, 24 + g, E.gpass * 8 + 7, l == 0);
+#endif
     };
     auto epilogue = [&](const Epi& E) {
       static_for<NPASS>([&](auto P_) { if ((int)P_ == E.pass) do_epilogue(P_, E); });
