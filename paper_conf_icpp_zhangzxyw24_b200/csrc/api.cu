@@ -890,12 +890,15 @@ int pretransformed_common(int is_deconv, int N, int H, int W, int C, int K, int 
   Plan pl;
   int rc = make_plan(N, H, W, C, K, R, S, pad_h, pad_w, is_deconv, &pl);
   if (rc != I2CW_OK) return rc;
-  if (pl.strip && pl.pair) {  // u has the filter-only (base) plan's layout (i2cw_filter_transform)
+  if (pl.strip) {  // u has the filter-only (base) plan's layout (i2cw_filter_transform)
     Plan pb;
     if ((rc = make_plan3(N, 1, H, W, C, K, 1, R, S, 0, pad_h, pad_w, is_deconv, 0, &pb, 2)) != I2CW_OK) return rc;
-    // the single-CTA strip kernel reads that layout and sums in the same order (bitwise equal)
-    if (!pb.pair && (rc = make_plan3(N, 1, H, W, C, K, 1, R, S, 0, pad_h, pad_w, is_deconv, 0, &pl, 4)) != I2CW_OK)
-      return rc;
+    if (pl.pair && !pb.pair) {
+      // the single-CTA strip kernel reads that layout and sums in the same order (bitwise equal)
+      if ((rc = make_plan3(N, 1, H, W, C, K, 1, R, S, 0, pad_h, pad_w, is_deconv, 0, &pl, 4)) != I2CW_OK) return rc;
+    } else if (!pl.pair && pb.pair) {
+      pl = pb;  // a strip plan too small for CTA pairs: the base kernel reads the pair layout
+    }
   }
   if ((rc = bind_device_of(x)) != I2CW_OK) return rc;
   auto matches = [&](const UTag& t) {

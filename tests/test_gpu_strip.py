@@ -66,3 +66,20 @@ def test_strip_k_chunks(kind):
         assert_parity(y, yr, b)
     finally:
         i2cw.debug_set_kchunk(old)
+
+
+def test_strip_pretransformed_layouts():
+    """A pre-transformed U is in the filter-only plan's layout: the CTA-pair layout for C = 512 (long
+    K loop), while a one-strip-group problem runs the single-CTA strip kernel in the one-shot call.
+    The '*' call then runs the base kernel on the pair layout; both match the oracle."""
+    cfg = ("conv", 1, 28, 20, 512, 64, 3, 3, 1, 1)
+    kind, N, H, W, C, K, R, S, ph, pw = cfg
+    p = i2cw.debug_plan(*cfg)
+    assert p["strip"] == 1 and p["pair"] == 0
+    x, w = inputs(kind, N, H, W, C, K, R, S)
+    y1, yr, b = run_case(*cfg)
+    u = i2cw.filter_transform(w.cuda())
+    y2 = i2cw.conv2d_nhwc_pretransformed(x.cuda(), u, K, R, S, ph, pw)
+    torch.cuda.synchronize()
+    assert_parity(y1, yr, b)
+    assert_parity(y2, yr, b)
