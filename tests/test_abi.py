@@ -147,3 +147,22 @@ def test_planner_concurrent_shapes():
     for t in ts:
         t.join()
     assert not errs, errs
+
+
+def test_strip_kernel_selection():
+    """The planner's measured rule (profiles/r02_strip_sweep.txt): the strip kernel
+    (CTA pairs) for the BASELINE configs with tall images (cfg2, cfg4-r5, cfg5a, cfg5b), the base
+    kernel for cfg3's 32x32 images, alpha = 12 and cfg4-r7; filter-only plans (the '*' layout)
+    never use it."""
+    strip = {"cfg2": ("conv", 128, 56, 56, 64, 64, 3, 3, 1, 1), "cfg4-r5": ("deconv", 64, 28, 28, 256, 256, 5, 5, 2, 2),
+             "cfg5a": ("conv", 256, 112, 112, 64, 64, 7, 7, 3, 3), "c64": ("conv", 256, 28, 28, 64, 64, 3, 3, 1, 1),
+             "c512": ("conv", 256, 28, 28, 512, 512, 3, 3, 1, 1)}
+    base = {"cfg3-r3": ("conv", 64, 32, 32, 128, 128, 3, 3, 1, 1), "cfg3-r9": ("conv", 64, 32, 32, 128, 128, 9, 9, 4, 4),
+            "cfg4-r7": ("deconv", 64, 28, 28, 256, 256, 7, 7, 3, 3)}
+    for name, cfg in strip.items():
+        p = i2cw.debug_plan(*cfg)
+        assert p["strip"] == 1 and p["pair"] == 1 and p["alpha"] == 8, name
+    for name, cfg in base.items():
+        assert i2cw.debug_plan(*cfg)["strip"] == 0, name
+    # i2cw_filter_bytes plans the filter alone (base layout): 2 alpha (ceil(K/64)*64) R ceil8(C) floats
+    assert i2cw.lib().i2cw_filter_bytes(64, 64, 3, 3) == 256 + 2 * 8 * 64 * 3 * 64 * 4
