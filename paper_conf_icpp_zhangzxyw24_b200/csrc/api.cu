@@ -578,10 +578,13 @@ int encode_y_map_strip(const Plan& pl, float* y, int L, CUtensorMap* map) {
   if (!enc) return I2CW_ECUDA;
   cuuint64_t dims[4] = {(cuuint64_t)pl.K, (cuuint64_t)pl.Q, (cuuint64_t)pl.P, (cuuint64_t)pl.N};
   cuuint64_t strides[3] = {(cuuint64_t)pl.K * 4, (cuuint64_t)pl.Q * pl.K * 4, (cuuint64_t)pl.P * pl.Q * pl.K * 4};
-  cuuint32_t box[4] = {16, (cuuint32_t)(L * pl.m), (cuuint32_t)pl.ROWS, 1};
-  cuuint32_t es[4] = {1, (cuuint32_t)pl.m, 1, 1};
+  // L = 2 is the warp-pair store box of the strip kernel (I2CW_STRIP_PAIRSTORE): 32 channels x 1
+  // column x ROWS rows, 128B swizzle (128-byte staging rows); L = 1: the per-warp 16-channel box
+  const bool pairbox = L == 2;
+  cuuint32_t box[4] = {pairbox ? 32u : 16u, pairbox ? 1u : (cuuint32_t)(L * pl.m), (cuuint32_t)pl.ROWS, 1};
+  cuuint32_t es[4] = {1, pairbox ? 1u : (cuuint32_t)pl.m, 1, 1};
   CUresult r = enc(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, y, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                   CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_NONE,
+                   pairbox ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_NONE,
                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   return r == CUDA_SUCCESS ? I2CW_OK : I2CW_EUNSUPPORTED;
 }

@@ -91,6 +91,9 @@ __device__ __forceinline__ void tmem_shift_up_warp(uint32_t taddr) {
 }
 
 constexpr int kStripLanes = 32;  // input rows per strip box (one TMEM subpartition)
+#ifndef I2CW_STRIP_PAIRSTORE
+#define I2CW_STRIP_PAIRSTORE 1  // warp pairs store 32-channel boxes (ym.m[1]); 0 = per-warp 16-channel boxes (ym.m[0])
+#endif
 #ifndef I2CW_STRIP_WARPSTORE
 #define I2CW_STRIP_WARPSTORE 1  // per-warp y stores (measured +1..3% over the warpgroup-run stores, 0)
 #endif
@@ -408,7 +411,78 @@ __global__ void __launch_bounds__(StripCfg<M, RW, PAIR>::NTHREADS, 1)
           }
         }
       });
-#if I2CW_STRIP_WARPSTORE
+#if I2CW_STRIP_WARPSTORE && I2CW_STRIP_PAIRSTORE
+      // Warp-pair stores: warps (g, sub) and (g ^ 1, sub) stage their 16-channel halves of the
+      // strip's rows into one [row][32 ch] buffer (128-byte rows, 128B swizzle, conflict-free) and
+      // the even warp issues one 32-channel box per column: half the TMA ops of per-warp stores,
+      // one 64-thread named barrier per column.
+      {
+        const bool mine = sub < nvalid;
+        Strip ms = strip_at(E.sg0 + (mine ? sub : 0));
+        const int gp = g >> 1, hh = g & 1;
+        const int pid = gp * 4 + sub;  // warp pair: named barrier 1 + pid, staging buffers
+        const bool lead = hh == 0;
+        uint8_t* pbase = o_smem + (size_t)pid * pl.NOB * 4096;
+        const uint32_t rbase = (uint32_t)(jr * 128);
+        const uint32_t rsw = (uint32_t)(jr & 7);
+        if (lead && lane32 == 0) {
+          bulk_wait_group_read_dyn(pl.NOB - 1);
+          if (PASS > 0 && !E.split) bulk_wait_group_all();  // this pair's pass-0 stores of the unit landed
+        }
+        named_bar_sync(1 + pid, 64);
+        const bool store = PASS == 0 && !E.split && !pl.ACCUM;
+        static_for<M>([&](auto I_) {
+          constexpr int i = I_;
+          const int ob = i % pl.NOB;
+          uint8_t* stg = pbase + (size_t)ob * 4096;
+#pragma unroll
+          for (int j = 0; j < CPW / 4; ++j) {
+            float2 o[2] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
+            static_for<GP / 2>([&](auto Q_) {
+              constexpr int idx0 = PASS * GP + 2 * (int)Q_;
+              constexpr int tl0 = 2 * (int)Q_;
+              if constexpr (idx0 == 0) {
+                constexpr float c0 = T::AT(i, 0), c1 = T::AT(i, A - 1);
+#pragma unroll
+                for (int e = 0; e < 2; ++e) {
+                  const float2 m0 = make_float2(mv[tl0][4 * j + 2 * e], mv[tl0][4 * j + 2 * e + 1]);
+                  const float2 m1 = make_float2(mv[tl0 + 1][4 * j + 2 * e], mv[tl0 + 1][4 * j + 2 * e + 1]);
+                  if constexpr (c0 != 0.f) o[e] = __ffma2_rn(make_float2(c0, c0), m0, o[e]);
+                  if constexpr (c1 != 0.f) o[e] = __ffma2_rn(make_float2(c1, c1), m1, o[e]);
+                }
+              } else {
+                constexpr float ca = T::AT(i, point_of(idx0, A));
+                constexpr int src = (i % 2 == 0) ? tl0 : tl0 + 1;
+#pragma unroll
+                for (int e = 0; e < 2; ++e) {
+                  const float2 mz = make_float2(mv[src][4 * j + 2 * e], mv[src][4 * j + 2 * e + 1]);
+                  if constexpr (ca == 1.f) o[e] = __fadd2_rn(o[e], mz);
+                  else if constexpr (ca != 0.f) o[e] = __ffma2_rn(make_float2(ca, ca), mz, o[e]);
+                }
+              }
+            });
+            if (out_row && mine)
+              *reinterpret_cast<float4*>(stg + rbase + ((((uint32_t)(hh * 4 + j)) ^ rsw) << 4)) =
+                  make_float4(o[0].x, o[0].y, o[1].x, o[1].y);
+          }
+          fence_proxy_async_smem();
+          // the buffer the next column writes was last read by column i + 1 - NOB
+          if (lead && lane32 == 0) bulk_wait_group_read_dyn(pl.NOB - 2);
+          named_bar_sync(1 + pid, 64);
+          if (lead && lane32 == 0) {
+            if (mine && !ABL(32)) {
+              if (store) tma_store_4d(&ym.m[1], stg, E.nb * NT + gp * 32, ms.tw * M + i, ms.rb * pl.ROWS, ms.n);
+              else tma_reduce_add_4d(&ym.m[1], stg, E.nb * NT + gp * 32, ms.tw * M + i, ms.rb * pl.ROWS, ms.n);
+            }
+            bulk_commit_group();
+          }
+        });
+        if (lead && lane32 == 0) bulk_wait_group_read<0>();
+        lt[6] += lclock() - le1;
+        lt[7] += 1;
+        return;
+      }
+#elif I2CW_STRIP_WARPSTORE
       // Per-warp stores: warp (g, sub) stages its own strip's rows (64-byte rows, 64B swizzle,
       // conflict-free) and its lane 0 issues that strip's box (16 channels x 1 tile x ROWS rows)
       // per output column -- no warpgroup barrier, each warp tracks its own bulk groups.
