@@ -419,8 +419,8 @@ def main():
                        "per_gpu_batch": N if args.scaling == "weak" else f"{N_cfg // world}-{-(-N_cfg // world)}",
                        "parallelism": f"batch-sharded x{world} (shard_range), no collective in the timed region",
                        "F(m,r)": f"F({p['m']},{S}) alpha={p['alpha']}",
-                       "kernel": ("fused_strip_kernel (CTA pairs)" if p.get("pair") else "fused_strip_kernel") if p.get("strip")
-                       else "fused_tc_kernel", "l2": "flushed (256 MiB memset) before every step",
+                       "kernel": ("fused_strip_kernel" if p.get("strip") else "fused_tc_kernel")
+                       + (" (CTA pairs)" if p.get("pair") else ""), "l2": "flushed (256 MiB memset) before every step",
                        "inputs": "x[n] ~ U[-1,1) seeded 1000+n per global image n (on device), w ~ U[-1,1) seed 7",
                        "step": f"i2cw_{'de' if is_deconv else ''}conv2d_nhwc (C ABI one-shot call: filter transform + fused kernel)"},
             "roofline": rf,

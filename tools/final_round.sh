@@ -1,7 +1,7 @@
 #!/bin/bash
 # Round-end style measurements: default bench line (as the driver runs it), the reference arm,
 # every BASELINE config through bench.py, clocks. Usage (under gpurun): bash tools/final_round.sh TAG
-TAG=${1:-r02}; OUT=gpurun_out; mkdir -p $OUT
+export TAG=${1:-r02}; OUT=gpurun_out; mkdir -p $OUT
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,power.draw --format=csv > $OUT/nvsmi_$TAG.txt
 python bench.py > $OUT/bench_cfg2_$TAG.json 2> $OUT/bench_cfg2_$TAG.err; tail -c 400 $OUT/bench_cfg2_$TAG.json; echo
 python bench.py --steps 20 --warmup 3 > $OUT/bench_cfg2_k20_$TAG.json 2>> $OUT/bench_cfg2_$TAG.err
