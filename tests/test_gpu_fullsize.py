@@ -29,9 +29,17 @@ def test_full_size_sampled(cfg):
     rng = np.random.default_rng(5)
     npts = 1500
     idx = np.stack([rng.integers(0, s, npts) for s in y.shape], 1)
-    # always include the last width column (boundary tile) and the last channel
+    # always include the last width column (boundary tile), the last channel, the first and last
+    # output rows (padding; the strip kernel's partial last row block) and the rows either side
+    # of every strip row-block boundary (halo lanes of the next strip)
     idx[:100, 2] = y.shape[2] - 1
     idx[100:200, 3] = y.shape[3] - 1
+    idx[200:300, 1] = y.shape[1] - 1
+    idx[300:350, 1] = 0
+    p = i2cw.debug_plan(kind, N, H, W, C, K, R, S, ph, pw)
+    edges = [e for rb in range(1, -(-y.shape[1] // p["ROWS"])) for e in (rb * p["ROWS"] - 1, rb * p["ROWS"])]
+    if p["strip"] and edges:
+        idx[350:550, 1] = np.asarray(edges)[rng.integers(0, len(edges), 200)]
     # only the images the sample touches go to the host
     imgs = np.unique(idx[:, 0])
     xs = x[torch.as_tensor(imgs, device="cuda")].cpu()
